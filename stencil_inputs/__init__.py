@@ -1,0 +1,279 @@
+"""Seeded synthetic inputs shared by the oracle tests and the CUDA path.
+
+This module holds NO arithmetic of the stencil method itself: it only draws
+fields and stencils. Both `oracle/` (through the tests) and the product path
+(through the tests and `bench.py`) consume what it produces; neither side imports
+the other.
+
+Contents
+--------
+* Counter-based field generator. Every value is a pure
+  function of (seed, global linear index), so any sub-box of a huge grid can be
+  regenerated independently. The CUDA runtime implements the *same* generator
+  on the device (`stencil_fill_field` in `include/stencil.h`); a GPU test checks
+  that the two agree bit for bit.
+* Stencil builders: star / box shapes ("star, box and cross",
+  orders 1-4) with the coefficient conventions of SURVEY §8(c) C-2.
+* Algorithm 1, the random stencil generator (§IV-B),
+  under the reading C-7 in DESIGN.md.
+
+Layouts: grids are row-major, slowest dimension first (``[nz][ny][nx]``, 2-D
+``[ny][nx]``). An access tensor of order r has shape ``(2r+1,)*ndim`` indexed
+``[dz+r][dy+r][dx+r]`` ("the neighbor points accessed and the central
+point are assigned a value of 1").
+"""
+from __future__ import annotations
+
+import itertools
+from typing import Dict, List, Sequence, Tuple
+
+import numpy as np
+
+# --------------------------------------------------------------------------
+# counter-based generator (C-3)
+# --------------------------------------------------------------------------
+_M64 = np.uint64(0xFFFFFFFFFFFFFFFF)
+_GOLDEN = np.uint64(0x9E3779B97F4A7C15)
+_SEEDMUL = np.uint64(0xD1B54A32D192ED03)
+
+KINDS = ("uniform12", "int1023")
+
+
+def mix64(x: np.ndarray) -> np.ndarray:
+    """splitmix64 output function applied to ``x + golden`` (wrapping uint64)."""
+    with np.errstate(over="ignore"):
+        z = (x + _GOLDEN).astype(np.uint64)
+        z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+        z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+        z = z ^ (z >> np.uint64(31))
+    return z
+
+
+def hash_index(seed: int, gidx: np.ndarray) -> np.ndarray:
+    """h(seed, g) = mix64((seed * 0xD1B54A32D192ED03) xor g)."""
+    with np.errstate(over="ignore"):
+        key = np.uint64(seed & 0xFFFFFFFFFFFFFFFF) * _SEEDMUL
+    return mix64(np.asarray(gidx, dtype=np.uint64) ^ key)
+
+
+def values_from_hash(h: np.ndarray, dtype: str, kind: str) -> np.ndarray:
+    """Map 64-bit hashes to field values.
+
+    ``uniform12``: exactly uniform in [1, 2): fp64 takes 52 mantissa bits
+    ``(h >> 12) | 0x3FF0...``, fp32 takes 23 bits ``(h >> 41) | 0x3F80...``.
+    ``int1023``: integers in [-1023, 1023] (``(h >> 53) % 2047 - 1023``), the
+    dyadic-exact pin P7 of SURVEY §8(c).
+    """
+    if kind == "uniform12":
+        if dtype == "f64":
+            bits = (h >> np.uint64(12)) | np.uint64(0x3FF0000000000000)
+            return bits.view(np.float64)
+        if dtype == "f32":
+            bits = ((h >> np.uint64(41)) | np.uint64(0x3F800000)).astype(np.uint32)
+            return bits.view(np.float32)
+    elif kind == "int1023":
+        v = ((h >> np.uint64(53)) % np.uint64(2047)).astype(np.int64) - 1023
+        return v.astype(np.float64 if dtype == "f64" else np.float32)
+    raise ValueError(f"bad dtype/kind {dtype}/{kind}")
+
+
+def make_field(dims: Sequence[int], seed: int, dtype: str = "f64", kind: str = "uniform12",
+               origin: Sequence[int] | None = None,
+               global_dims: Sequence[int] | None = None) -> np.ndarray:
+    """Field of shape ``dims`` whose element at local index i is
+    ``value(h(seed, g))`` with g the row-major linear index of ``origin + i``
+    inside ``global_dims`` (default: the box is the whole grid)."""
+    dims = tuple(int(d) for d in dims)
+    gdims = tuple(int(d) for d in (global_dims or dims))
+    org = tuple(int(o) for o in (origin or (0,) * len(dims)))
+    assert len(gdims) == len(dims) == len(org)
+    strides = np.ones(len(dims), dtype=np.uint64)
+    for k in range(len(dims) - 2, -1, -1):
+        strides[k] = strides[k + 1] * np.uint64(gdims[k + 1])
+    gidx = np.zeros(dims, dtype=np.uint64)
+    for k, (n, o) in enumerate(zip(dims, org)):
+        shape = [1] * len(dims)
+        shape[k] = n
+        gidx = gidx + (np.arange(o, o + n, dtype=np.uint64) * strides[k]).reshape(shape)
+    return values_from_hash(hash_index(seed, gidx), dtype, kind)
+
+
+# --------------------------------------------------------------------------
+# stencil builders (P:L85 shapes; coefficients per C-2)
+# --------------------------------------------------------------------------
+
+def _empty(ndim: int, r: int):
+    shape = (2 * r + 1,) * ndim
+    return np.zeros(shape, dtype=np.uint8), np.zeros(shape, dtype=np.float64)
+
+
+def star(ndim: int, r: int, centre: float, arm: Sequence[float]):
+    """Star of order r: centre plus +-k along each axis, weight ``arm[k-1]``."""
+    acc, c = _empty(ndim, r)
+    ctr = (r,) * ndim
+    acc[ctr] = 1
+    c[ctr] = centre
+    for ax in range(ndim):
+        for k in range(1, r + 1):
+            for s in (-1, 1):
+                idx = list(ctr)
+                idx[ax] += s * k
+                acc[tuple(idx)] = 1
+                c[tuple(idx)] = arm[k - 1]
+    return acc, c
+
+
+def box(ndim: int, r: int, centre: float, other: float):
+    acc, c = _empty(ndim, r)
+    acc[...] = 1
+    c[...] = other
+    c[(r,) * ndim] = centre
+    return acc, c
+
+
+def heat2d():
+    """C1: 2-D 5-point heat, alpha = 1/8 -> centre 1/2, arms 1/8 (dyadic)."""
+    return star(2, 1, 0.5, [0.125])
+
+
+def heat3d():
+    """C2: 3-D 7-point heat, alpha = 1/8 -> centre 1/4, arms 1/8 (dyadic)."""
+    return star(3, 1, 0.25, [0.125])
+
+
+def star25():
+    """C3: order-4 3-D star, arm weights 1/16, 1/32, 1/64, 1/128, centre 19/64."""
+    return star(3, 4, 19.0 / 64.0, [1 / 16, 1 / 32, 1 / 64, 1 / 128])
+
+
+def box125():
+    """C4: order-2 3-D box, 124 x 1/128 plus centre 4/128."""
+    return box(3, 2, 4.0 / 128.0, 1.0 / 128.0)
+
+
+# --------------------------------------------------------------------------
+# Algorithm 1 under reading C-7
+# --------------------------------------------------------------------------
+
+def ring_index(offset: Sequence[int]) -> int:
+    """Chebyshev ring of an offset (order = max extent, Table II)."""
+    return max(abs(int(v)) for v in offset)
+
+
+def _moore(p: Tuple[int, ...]) -> List[Tuple[int, ...]]:
+    out = []
+    for d in itertools.product((-1, 0, 1), repeat=len(p)):
+        if any(d):
+            out.append(tuple(a + b for a, b in zip(p, d)))
+    return out
+
+
+def random_stencil(ndim: int, order: int, seed: int, p: float = 0.5):
+    """Algorithm 1: iteratively sample neighbours of the previous order's
+    selected points, delete rings order-1 and order-2, append the set.
+
+    Returns ``(access, npList)``; ``npList[k-1]`` is the set selected at order k.
+    ``random()`` is an independent Bernoulli(p) draw per candidate, redrawn until
+    at least one ring-``order`` point is kept (so the stencil order is exactly N).
+    """
+    if not (1 <= order <= 4) or ndim not in (2, 3):
+        raise ValueError("order in 1..4, ndim in {2,3}")
+    rng = np.random.Generator(np.random.PCG64(seed))
+    centre = (0,) * ndim
+    np_list: List[set] = []
+    prev = {centre}
+    for k in range(1, order + 1):
+        cand = set()
+        for q in sorted(prev):
+            cand.update(_moore(q))
+        if k >= 2:
+            cand = {q for q in cand if ring_index(q) != k - 1}          # delete(neighbor_{k-1})
+        if k > 2:
+            cand = {q for q in cand if ring_index(q) != k - 2}          # delete(neighbor_{k-2})
+        cand_sorted = sorted(cand)
+        while True:
+            keep = rng.random(len(cand_sorted)) < p
+            sel = {q for q, kk in zip(cand_sorted, keep) if kk}
+            if any(ring_index(q) == k for q in sel):
+                break
+        np_list.append(sel)
+        prev = sel
+    acc = np.zeros((2 * order + 1,) * ndim, dtype=np.uint8)
+    acc[(order,) * ndim] = 1
+    for s in np_list:
+        for q in s:
+            acc[tuple(v + order for v in q)] = 1
+    return acc, np_list
+
+
+def random_coeffs(access: np.ndarray, seed: int) -> np.ndarray:
+    """C5 coefficients: U(0,1) on the accessed entries, normalised to sum 1."""
+    rng = np.random.Generator(np.random.PCG64(seed ^ 0x5EED))
+    c = np.where(access != 0, rng.random(access.shape), 0.0)
+    return c / c.sum()
+
+
+def config_stencil(name: str, seed: int = 0):
+    """Named workloads of BASELINE.json configs."""
+    if name == "heat2d":
+        return heat2d()
+    if name == "heat3d":
+        return heat3d()
+    if name == "star25":
+        return star25()
+    if name == "box125":
+        return box125()
+    if name.startswith("random3d"):
+        # random3d:<order>:<seed>
+        _, order, s = name.split(":")
+        acc, _ = random_stencil(3, int(order), int(s))
+        return acc, random_coeffs(acc, int(s))
+    raise KeyError(name)
+
+
+# --------------------------------------------------------------------------
+# closed-form pin fields; inputs only, no stencil arithmetic
+# --------------------------------------------------------------------------
+
+def linear_field(dims: Sequence[int], a: Sequence[float], b: float) -> np.ndarray:
+    grids = np.meshgrid(*[np.arange(n, dtype=np.float64) for n in dims], indexing="ij")
+    return sum(ak * g for ak, g in zip(a, grids)) + b
+
+
+def eigenmode_field(dims: Sequence[int], modes: Sequence[int]) -> np.ndarray:
+    """prod_k sin(pi m_k i_k / (n_k - 1)); zero on the outer faces."""
+    out = np.ones(tuple(dims), dtype=np.float64)
+    for k, (n, m) in enumerate(zip(dims, modes)):
+        shape = [1] * len(dims)
+        shape[k] = n
+        out = out * np.sin(np.pi * m * np.arange(n) / (n - 1)).reshape(shape)
+    return out
+
+
+def cosine_field(dims: Sequence[int], wave: Sequence[float], phase: float) -> np.ndarray:
+    grids = np.meshgrid(*[np.arange(n, dtype=np.float64) for n in dims], indexing="ij")
+    return np.cos(sum(k * g for k, g in zip(wave, grids)) + phase)
+
+
+def dyadic_random_stencil(ndim: int, order: int, seed: int):
+    """A random Alg.1 pattern with coefficients k_o / 2^m, integer k_o in
+    [-3, 3] \\ {0} and m = ceil(log2 sum|k_o|) so that sum |c_o| <= 1 (pin P7:
+    with integer |u_0| <= 1023 every partial sum is exact while 10 + m*T <= 53
+    in fp64 or <= 24 in fp32). Returns ``(access, coeffs, m)``."""
+    acc, _ = random_stencil(ndim, order, seed)
+    rng = np.random.Generator(np.random.PCG64(seed + 77))
+    nnz = int(acc.sum())
+    ks = rng.integers(1, 4, size=nnz) * np.where(rng.random(nnz) < 0.3, -1, 1)
+    m = int(np.ceil(np.log2(np.abs(ks).sum())))
+    c = np.zeros(acc.shape)
+    c[acc != 0] = ks / float(2 ** m)
+    return acc, c, m
+
+
+CONFIGS: Dict[str, dict] = {
+    "C1": dict(ndim=2, dims=(256, 256), stencil="heat2d", dtype="f64", steps=10, seed=0xC0FFEE + 1),
+    "C2": dict(ndim=3, dims=(512, 512, 512), stencil="heat3d", dtype="f64", steps=10, seed=0xC0FFEE + 2),
+    "C3": dict(ndim=3, dims=(768, 768, 768), stencil="star25", dtype="f32", steps=10, seed=0xC0FFEE + 3),
+    "C4": dict(ndim=3, dims=(512, 512, 512), stencil="box125", dtype="f64", steps=10, seed=0xC0FFEE + 4),
+    "C5": dict(ndim=3, dims=(1024, 1024, 1024), stencil="random3d", dtype="f64", steps=4, seed=0xC0FFEE + 5),
+}
