@@ -1,0 +1,258 @@
+/*
+ * include/stencil.h -- C ABI of the B200-native StencilMART hot path.
+ *
+ * StencilMART (Sun et al., IPDPS'22; /root/reference/PAPER.md, cited "P:L<line>")
+ * profiles every stencil under every optimization combination (OC) to label
+ * the best one: "the performance of each stencil input is profiled with
+ * different OCs on the target GPU, and the OC with the best performance is
+ * labeled. Specifically, the StencilMART randomly searches the parameter
+ * settings under each OC and selects the shortest execution time" (P:L119,
+ * §IV-A; also P:L234, §V-A.2). This library is that data-parallel path: the
+ * sweep of one arbitrary 2-D/3-D stencil under any OC of Table I, and the
+ * per-OC timing sweep that produces the label.
+ *
+ * Conventions shared by every entry point
+ * ---------------------------------------
+ * - Every function returns a stencil_status_t (0 = OK, < 0 = error) unless
+ *   stated otherwise; the thread-local message of the last error is returned by
+ *   stencil_last_error().
+ * - Grids are dense, row-major, slowest dimension first: 3-D [nz][ny][nx],
+ *   2-D [ny][nx] (x contiguous), element type per stencil_dtype_t.
+ * - Device pointers are owned by the caller (PyTorch in the Python binding),
+ *   must be at least 16-byte aligned and hold the whole grid. Host pointers
+ *   (stencil_run_host) are plain caller memory.
+ * - Argument validation happens before any CUDA call, so invalid arguments are
+ *   reported as STENCIL_E_INVAL / STENCIL_E_OC_INVALID even without a GPU.
+ * - Work is enqueued on the plan's stream (stencil_plan_set_stream; default:
+ *   the legacy default stream) and is asynchronous w.r.t. the host unless
+ *   stated otherwise. CUDA errors are reported by the call that detects them.
+ * - A plan must not be used concurrently from several host threads; distinct
+ *   plans are independent.
+ */
+#ifndef STENCILMART_STENCIL_H
+#define STENCILMART_STENCIL_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define STENCIL_ABI_VERSION 1
+
+/* Opaque plan: one stencil on one grid shape under one OC and parameter
+ * setting. Created by stencil_plan_create, owned by the caller, released by
+ * stencil_plan_destroy. It owns its compiled kernels, TMA descriptors, events
+ * and (multi-GPU) its NCCL communicator. */
+typedef struct stencil_plan_s *stencil_plan_t;
+
+typedef enum { STENCIL_F32 = 0, STENCIL_F64 = 1 } stencil_dtype_t;
+
+/* OC bitmask (Table I). OC id = OR of these bits; 0 is the
+ * plain kernel ("each GPU thread works on a single output point").
+ * Table I constraints: BM and CM are mutually exclusive; RT and PR are only
+ * valid with ST. Exactly 30 ids are valid (6 without ST, 24 with ST). */
+enum {
+    STENCIL_OC_ST = 1,   /* streaming (2.5-D blocking, concurrent streaming) */
+    STENCIL_OC_BM = 2,   /* block merging: k adjacent outputs per thread */
+    STENCIL_OC_CM = 4,   /* cyclic merging: k outputs a fixed distance apart */
+    STENCIL_OC_RT = 8,   /* retiming: per-plane partial sums */
+    STENCIL_OC_PR = 16,  /* prefetching: next plane loaded during compute */
+    STENCIL_OC_TB = 32   /* temporal blocking: T fused time steps */
+};
+#define STENCIL_NUM_OC 30
+
+typedef enum {
+    STENCIL_OK = 0,
+    STENCIL_E_INVAL = -1,          /* bad argument (dims, order, access, coeffs, dtype, pointers) */
+    STENCIL_E_OC_INVALID = -2,     /* OC violates Table I */
+    STENCIL_E_OC_INFEASIBLE = -3,  /* OC + setting exceeds a hardware limit (the paper's OC "crash") */
+    STENCIL_E_NOMEM = -4,
+    STENCIL_E_CUDA = -5,
+    STENCIL_E_NCCL = -6,
+    STENCIL_E_NVRTC = -7,          /* kernel specialisation failed */
+    STENCIL_E_STATE = -8           /* call not valid in the plan's current state (e.g. no workspace) */
+} stencil_status_t;
+
+/* Parameter setting of an OC (§IV-E: numeric parameters are powers of
+ * two, Boolean parameters are {0,1}, enumerations start at 1). A field equal to
+ * 0 (-1 for smem) selects the library default for the OC and dtype; fields an
+ * OC does not use are ignored. */
+typedef struct {
+    int32_t smem;         /* Boolean "shared memory usage"; OCs base/BM/CM only:
+                             1 = stage an (x,y,z) tile + halo in shared memory, 0 = global loads */
+    int32_t bx;           /* CTA tile width along x in outputs (power of two, 8..256) */
+    int32_t by;           /* threads per CTA along y (power of two) */
+    int32_t bz;           /* non-streaming tiled kernels: output planes per CTA */
+    int32_t vx;           /* outputs per thread along x (1, 2, 4): one 128-bit vector */
+    int32_t merge;        /* BM/CM merge factor k (outputs per thread along y; 1..8) */
+    int32_t stream_chunk; /* ST: output planes per CTA ("concurrent streaming") */
+    int32_t tb_steps;     /* TB: time steps fused per launch (2..8) */
+    int32_t pr_stages;    /* PR: planes in flight in the TMA pipeline (2..4) */
+    int32_t reserved[3];  /* must be 0 */
+} stencil_params_t;
+
+/* Read-only facts about a plan (for tests, reports and the sweep). */
+typedef struct {
+    int32_t ndim, order, nnz, dtype;
+    int32_t ext[6];           /* z_lo, z_hi, y_lo, y_hi, x_lo, x_hi: neighbour extents (<= order) */
+    uint32_t oc;
+    stencil_params_t params;  /* the resolved setting (defaults filled in) */
+    int32_t kernel_family;    /* 0 naive, 1 tiled, 2 stream, 3 stream+TB */
+    int32_t smem_bytes;       /* dynamic shared memory per CTA */
+    int32_t threads;          /* threads per CTA */
+    int32_t regs;             /* registers per thread of the main kernel (0 until compiled) */
+    int32_t uses_tma;         /* 1 if halo tiles are staged with cp.async.bulk.tensor */
+    int64_t points;           /* interior points updated per time step (global grid) */
+    char kernel_name[128];    /* lowered name of the main kernel */
+} stencil_plan_info_t;
+
+/* ---------------------------------------------------------------------------
+ * Plan lifetime
+ * ------------------------------------------------------------------------- */
+
+/* Create a plan (§8(a) rows a1-a3 of SURVEY.md).
+ *   ndim    2 or 3.
+ *   dims    ndim extents, slowest first ([nz,ny,nx] or [ny,nx]); each >= 2*order+1.
+ *           With a communicator set later, dims[0] is the LOCAL slab depth.
+ *   order   r in 1..4: frame width and access-tensor radius (order = maximum
+ *           extent of the neighbours).
+ *   access  uint8[(2r+1)^ndim], row-major [dz+r][dy+r][dx+r]; 1 = accessed.
+ *           The centre must be 1; the maximum extent may be < r.
+ *   coeffs  double[(2r+1)^ndim], same layout; must be 0 where access == 0.
+ *           Rounded to the plan dtype once, round-to-nearest-even.
+ *   dtype   STENCIL_F32 or STENCIL_F64 (arithmetic type of the sweep).
+ *   oc      OC bitmask; STENCIL_E_OC_INVALID if it violates Table I.
+ *   params  NULL = defaults.
+ * The update computed by every OC is
+ *   u_{t+1}[p] = sum_{o in S} c_o u_t[p+o]   for r <= p_k < n_k - r on every axis,
+ *   u_{t+1}[p] = u_t[p]                     elsewhere (the frame; C-1),
+ * each sum evaluated as one fused-multiply-add chain in lexicographic
+ * (dz,dy,dx) order, so every OC returns bitwise the same grid.
+ * Kernel specialisation (NVRTC, sm_100a) happens here; the result is cached
+ * per process and, if STENCIL_CACHE_DIR (default ~/.cache/stencilmart) is
+ * writable, on disk. Needs a CUDA device for the compile+load step unless the
+ * environment variable STENCIL_DEFER_COMPILE=1 is set (compile at first run). */
+int stencil_plan_create(stencil_plan_t *plan, int ndim, const int64_t *dims, int order,
+                        const uint8_t *access, const double *coeffs, stencil_dtype_t dtype,
+                        uint32_t oc, const stencil_params_t *params);
+
+/* Release the plan and everything it owns. NULL is a no-op. */
+void stencil_plan_destroy(stencil_plan_t plan);
+
+/* Stream on which stencil_run / stencil_oc_sweep enqueue work (a cudaStream_t). */
+int stencil_plan_set_stream(stencil_plan_t plan, void *cuda_stream);
+
+/* Bytes of device workspace stencil_run needs for steps >= 2 (one grid). */
+size_t stencil_plan_workspace_bytes(stencil_plan_t plan);
+
+/* Caller-owned device workspace (>= stencil_plan_workspace_bytes, 16-B aligned).
+ * Must stay valid while the plan runs. */
+int stencil_plan_set_workspace(stencil_plan_t plan, void *dev_ptr, size_t bytes);
+
+/* Fill *info. Host-only. */
+int stencil_plan_info(stencil_plan_t plan, stencil_plan_info_t *info);
+
+/* ---------------------------------------------------------------------------
+ * Sweeps
+ * ------------------------------------------------------------------------- */
+
+/* Advance `steps` (>= 0) time steps: out = S^steps(in). `in` is preserved;
+ * in != out (STENCIL_E_INVAL otherwise); steps == 0 copies. steps >= 2 needs a
+ * workspace. The frame of `in` is copied once into out (and the workspace);
+ * TB OCs launch ceil(steps/T) times, the last launch fusing the remainder. */
+int stencil_run(stencil_plan_t plan, const void *in_dev, void *out_dev, int steps);
+
+/* End-to-end form: `in_host` / `out_host` are host buffers of the grid. The
+ * call copies in_host to device buffers it owns, runs `steps` steps with the
+ * plan's OC, copies the result back and synchronises the plan's stream. */
+int stencil_run_host(stencil_plan_t plan, const void *in_host, void *out_host, int steps);
+
+/* The label generator: for each of the 30 OCs in ascending id
+ * order and each of `settings_per_oc` parameter settings (the plan's own
+ * setting's defaults first, then seeded random powers of two, see
+ * stencil_sample_params), create a plan for the same stencil, run one warm-up,
+ * then `reps` timed runs of `steps` steps with CUDA events on the plan's
+ * stream; the setting's time is the median, the OC's time the minimum over its
+ * settings. Infeasible OCs get +INF. best_oc = argmin over finite times, ties
+ * to the smallest id. With a communicator, per-OC times are the max over ranks
+ * (all ranks return identical vectors). `in` is preserved, `out` receives the
+ * last run's result. Outputs:
+ *   times_ms[30], oc_ids[30] (ascending), best_params[30], *best_oc.
+ * Synchronises the plan's stream. */
+int stencil_oc_sweep(stencil_plan_t plan, const void *in_dev, void *out_dev, int steps,
+                     int settings_per_oc, int reps, uint64_t seed,
+                     float *times_ms, uint32_t *oc_ids, stencil_params_t *best_params,
+                     uint32_t *best_oc);
+
+/* ---------------------------------------------------------------------------
+ * OC lattice and parameter space (host only, no GPU needed)
+ * ------------------------------------------------------------------------- */
+
+/* 1 if `oc` satisfies Table I, else 0. */
+int stencil_oc_valid(uint32_t oc);
+
+/* Write the 30 valid OC ids in ascending order into ids[30]; returns 30. */
+int stencil_oc_list(uint32_t *ids);
+
+/* Static name of an OC ("base", "ST", "TB_CM", "ST_BM_RT_PR", ...: components in
+ * the order ST, TB, BM, CM, RT, PR); NULL for an invalid id. */
+const char *stencil_oc_name(uint32_t oc);
+
+/* The k-th (k >= 0) sampled setting for `oc` under `seed`: k = 0 is the
+ * default setting, k >= 1 draws each numeric field as a power of two from the
+ * OC's range with a counter-based hash of (seed, oc, k). Deterministic. */
+int stencil_sample_params(uint32_t oc, int ndim, stencil_dtype_t dtype, uint64_t seed, int k,
+                          stencil_params_t *out);
+
+/* ---------------------------------------------------------------------------
+ * Synthetic inputs (the counter-based generator of DESIGN.md, reading C-3)
+ * ------------------------------------------------------------------------- */
+
+/* Fill a device box of shape box_dims (ndim values, slowest first) whose
+ * element i holds value(h(seed, g)), g = the row-major linear index of
+ * (origin + i) in a grid of shape global_dims. kind 0 = uniform in [1,2),
+ * kind 1 = integers in [-1023, 1023]. Enqueued on `cuda_stream`. */
+int stencil_fill_field(void *dev_ptr, stencil_dtype_t dtype, int ndim, const int64_t *box_dims,
+                       const int64_t *origin, const int64_t *global_dims, uint64_t seed, int kind,
+                       void *cuda_stream);
+
+/* ---------------------------------------------------------------------------
+ * Multi-GPU (one process per GPU; grids slab-decomposed along dims[0])
+ * ------------------------------------------------------------------------- */
+
+/* Fill id[128] with a fresh NCCL unique id (call on rank 0, broadcast it). */
+int stencil_nccl_unique_id(uint8_t *id);
+
+/* Attach the plan to a communicator of `nranks` ranks. The plan's grid becomes
+ * rank `rank`'s slab: dims[0] local planes of a global grid whose depth is the
+ * sum over ranks; the frame exists only at the global faces. Buffers passed to
+ * stencil_run then hold only the local slab; halo planes are exchanged with
+ * ranks +-1 every step (every T steps for TB) with ncclSend/ncclRecv on the
+ * plan's stream, overlapped with the interior sweep. Collective: all ranks call
+ * it with the same id. */
+int stencil_plan_set_comm(stencil_plan_t plan, const uint8_t *id, int rank, int nranks);
+
+/* Slab layout of `rank` among `nranks` for a global depth nz_global: writes
+ * {z_begin, z_end} of the rank's slab (near-equal split). Host only. */
+int stencil_slab_range(int64_t nz_global, int rank, int nranks, int64_t *z_begin, int64_t *z_end);
+
+/* ---------------------------------------------------------------------------
+ * Diagnostics
+ * ------------------------------------------------------------------------- */
+
+/* Thread-local message of the last error (empty string if none). */
+const char *stencil_last_error(void);
+
+/* Number of kernels this library launched in this process so far (for the
+ * benchmark's gpu_launches count). */
+uint64_t stencil_launch_count(void);
+
+/* STENCIL_ABI_VERSION of the loaded library. */
+int stencil_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* STENCILMART_STENCIL_H */

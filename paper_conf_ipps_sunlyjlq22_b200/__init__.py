@@ -1,0 +1,14 @@
+"""B200-native StencilMART hot path (Sun et al., IPDPS'22).
+
+The sweep of an arbitrary generated 2-D/3-D stencil under every optimization
+combination (OC) of Table I, and the per-OC timing sweep that labels the best
+OC. Compute lives in libstencilmart.so (C ABI: include/stencil.h); this package
+is its thin ctypes binding.
+"""
+from .binding import (F32, F64, NUM_OC, OC_BM, OC_CM, OC_PR, OC_RT, OC_ST, OC_TB, Plan, StencilError,
+                      exported_symbols, fill_field, gstencil_per_s, launch_count, lib, nccl_unique_id,
+                      oc_from_name, oc_list, oc_name, oc_valid, sample_params, slab_range)
+
+__all__ = ["F32", "F64", "NUM_OC", "OC_BM", "OC_CM", "OC_PR", "OC_RT", "OC_ST", "OC_TB", "Plan",
+           "StencilError", "exported_symbols", "fill_field", "gstencil_per_s", "launch_count", "lib",
+           "nccl_unique_id", "oc_from_name", "oc_list", "oc_name", "oc_valid", "sample_params", "slab_range"]

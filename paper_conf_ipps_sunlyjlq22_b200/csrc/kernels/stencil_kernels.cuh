@@ -1,0 +1,573 @@
+// stencil_kernels.cuh -- hand-written sm_100a kernel templates, one family per
+// optimization combination (OC) of StencilMART Table I.
+//
+// This header is compiled at plan-creation time by NVRTC (runtime/codegen.cpp)
+// together with a generated stencil descriptor `S` that bakes in the offsets
+// and coefficients of one stencil (the paper generates "stencil programs",
+// P:L25). The descriptor holds only data; all logic is here.
+//
+// Descriptor contract (generated):
+//   typedef <float|double> T;
+//   static constexpr int NNZ, ZLO, ZHI, YLO, YHI, XLO, XHI, NZ, NY, NX;
+//       neighbour extents: dz in [-ZLO, ZHI], NZ = ZLO + ZHI + 1, etc.
+//   static __device__ constexpr int idx(int zi, int yi, int xi);
+//       coefficient index of offset (zi-ZLO, yi-YLO, xi-XLO) or -1 if not accessed;
+//       indices are the lexicographic (dz,dy,dx) rank of the offset.
+//   static __device__ constexpr T coef(int i);
+//   static constexpr int NOPS; static __device__ constexpr unsigned op(int i);
+//       the variant's op table (see run_gather / run_scatter).
+//
+// Arithmetic contract (SURVEY C-4): every output
+// is ONE fused-multiply-add chain acc = fma(c_o, u[p+o], acc) starting from 0
+// over the offsets in lexicographic (dz,dy,dx) order. Every kernel below keeps
+// that order per output, so all OCs produce bitwise identical grids.
+//
+// Frame rule (C-1): points outside the update box keep their value;
+// kernels only write outputs inside the compute box (a sub-box of the update
+// box); the frame of the output buffer is copied once by the runtime.
+
+namespace smart {
+
+typedef long long i64;
+
+struct alignas(64) TmaDesc { unsigned long long v[16]; };   // CUtensorMap, opaque
+
+struct Grid {
+  int nz, ny, nx;                    // array extents (elements)
+  i64 sy, sz;                        // element strides of y and z
+  int uz0, uz1, uy0, uy1, ux0, ux1;  // update box: points inside are updated
+  int cz0, cz1, cy0, cy1, cx0, cx1;  // compute box: outputs written by this launch
+  int vec_ok;                        // 1 if rows are VX-aligned (vector stores allowed)
+};
+
+// ---------------------------------------------------------------------------
+// small PTX helpers
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ unsigned smem_u32(const void* p) {
+  return static_cast<unsigned>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(unsigned long long* bar, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;"
+               :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@!P1 bra WAIT_%=;\n\t}"
+      :: "r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void tma_load_3d(void* dst, const TmaDesc* desc, unsigned long long* bar,
+                                            int x, int y, int z) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%2, %3, %4}], [%5];"
+      :: "r"(smem_u32(dst)), "l"(reinterpret_cast<unsigned long long>(desc)),
+         "r"(x), "r"(y), "r"(z), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void tma_prefetch_desc(const TmaDesc* desc) {
+  asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<unsigned long long>(desc)) : "memory");
+}
+template <int BYTES>
+__device__ __forceinline__ void cp_async_zfill(void* dst, const void* src, bool valid) {
+  static_assert(BYTES == 4 || BYTES == 8 || BYTES == 16, "cp.async size");
+  asm volatile("cp.async.ca.shared.global [%0], [%1], %2, %3;"
+               :: "r"(smem_u32(dst)), "l"(src), "n"(BYTES), "r"(valid ? BYTES : 0) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" :: "n"(N) : "memory"); }
+
+// ---------------------------------------------------------------------------
+// vector access: VX consecutive elements, 128-bit (or 64-bit) accesses
+// ---------------------------------------------------------------------------
+template <class T, int VX> struct Vec { T e[VX]; };
+
+template <class T, int VX>
+__device__ __forceinline__ void lds_vec(const T* p, T (&w)[VX]) {
+  if constexpr (sizeof(T) * VX == 16) {
+    const float4 q = *reinterpret_cast<const float4*>(p);
+    const T* t = reinterpret_cast<const T*>(&q);
+#pragma unroll
+    for (int e = 0; e < VX; ++e) w[e] = t[e];
+  } else if constexpr (sizeof(T) * VX == 32) {
+    const float4 q0 = reinterpret_cast<const float4*>(p)[0];
+    const float4 q1 = reinterpret_cast<const float4*>(p)[1];
+    const T* t0 = reinterpret_cast<const T*>(&q0);
+    const T* t1 = reinterpret_cast<const T*>(&q1);
+#pragma unroll
+    for (int e = 0; e < VX / 2; ++e) { w[e] = t0[e]; w[e + VX / 2] = t1[e]; }
+  } else if constexpr (sizeof(T) * VX == 8) {
+    const float2 q = *reinterpret_cast<const float2*>(p);
+    const T* t = reinterpret_cast<const T*>(&q);
+#pragma unroll
+    for (int e = 0; e < VX; ++e) w[e] = t[e];
+  } else {
+#pragma unroll
+    for (int e = 0; e < VX; ++e) w[e] = p[e];
+  }
+}
+
+template <class T, int VX>
+__device__ __forceinline__ void stg_vec(T* p, const T (&w)[VX]) {
+  if constexpr (sizeof(T) * VX == 16) {
+    float4 q;
+    T* t = reinterpret_cast<T*>(&q);
+#pragma unroll
+    for (int e = 0; e < VX; ++e) t[e] = w[e];
+    *reinterpret_cast<float4*>(p) = q;
+  } else if constexpr (sizeof(T) * VX == 8) {
+    float2 q;
+    T* t = reinterpret_cast<T*>(&q);
+#pragma unroll
+    for (int e = 0; e < VX; ++e) t[e] = w[e];
+    *reinterpret_cast<float2*>(p) = q;
+  } else {
+#pragma unroll
+    for (int e = 0; e < VX; ++e) p[e] = w[e];
+  }
+}
+
+__device__ __forceinline__ double fma_t(double a, double b, double c) { return __fma_rn(a, b, c); }
+__device__ __forceinline__ float fma_t(float a, float b, float c) { return __fmaf_rn(a, b, c); }
+
+// ---------------------------------------------------------------------------
+// compile-time pattern predicates (fold to constants after unrolling)
+// ---------------------------------------------------------------------------
+template <class S>
+__device__ __forceinline__ constexpr int cidx(int zi, int yi, int xi) {
+  return (zi < 0 || zi >= S::NZ || yi < 0 || yi >= S::NY || xi < 0 || xi >= S::NX) ? -1
+                                                                                   : S::idx(zi, yi, xi);
+}
+
+// compile-time loop: f(IC<B>{}), ..., f(IC<E-1>{})
+template <int V> struct IC { static constexpr int value = V; };
+template <int B, int E, class F>
+__device__ __forceinline__ void static_for(F&& f) {
+  if constexpr (B < E) {
+    f(IC<B>{});
+    static_for<B + 1, E>(f);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Window loaders.  `get(j, kv, w)` fills w[VX] with the elements at relative
+// row j and columns [kv*VX, kv*VX+VX) of one plane.
+// ---------------------------------------------------------------------------
+template <class T, int VX, int LD>
+struct SmemPlane {                    // shared memory, compile-time row pitch
+  const T* p;                          // element (row 0, col 0) of this thread
+  __device__ __forceinline__ void get(int j, int kv, T (&w)[VX]) const {
+    lds_vec<T, VX>(p + j * LD + kv * VX, w);
+  }
+};
+
+template <class T, int VX, int NROW>
+struct GlobalPlane {                  // global memory through the read-only path
+  const T* p;                          // element (plane z+dz, col 0) -- rows via rowoff
+  const i64* rowoff;                   // NROW clamped row offsets, index j + YLO
+  int yshift;                          // = YLO
+  __device__ __forceinline__ void get(int j, int kv, T (&w)[VX]) const {
+    const T* q = p + rowoff[j + yshift] + kv * VX;
+#pragma unroll
+    for (int e = 0; e < VX; ++e) w[e] = __ldg(q + e);
+  }
+};
+
+// ---------------------------------------------------------------------------
+// Compute on a thread tile of M rows x VX columns, driven by the op table of
+// the generated descriptor (S::NOPS, S::op(i); built by runtime/codegen.cpp).
+//   BM: outputs at rows 0..M-1 (adjacent, "block merging").
+//   CM: output m at row m*BY (a fixed distance, "cyclic merging").
+// An op is either a window LOAD of VX consecutive values of one plane, or an
+// FMA of one loaded value into one accumulator:
+//   LOAD (bit31 = 0): zi = op & 15, row j = ((op >> 4) & 255) - 128,
+//                     vector kv = ((op >> 12) & 15) - 8  (columns [kv*VX, kv*VX+VX))
+//   FMA  (bit31 = 1): coefficient id = op & 1023, element e = (op >> 10) & 3,
+//                     output column v = (op >> 12) & 3, output row m = (op >> 14) & 7,
+//                     slice zi = (op >> 17) & 15
+// The generator emits each value once per window and, per accumulator, the
+// FMAs in lexicographic (dz, dy, dx) order.
+// run_gather:  out plane z reads plane z + zi - ZLO through pl[zi].
+// run_scatter: retiming. pl is input plane p; slice zi adds into the
+//              partial sums of output plane p - (zi - ZLO), kept in
+//              acc[(U + NZ - zi) % NZ] (a register queue rotated at compile time).
+// ---------------------------------------------------------------------------
+template <class S, int VX, int M, class L>
+__device__ __forceinline__ void run_gather(const L (&pl)[S::NZ], typename S::T (&acc)[M][VX]) {
+  typedef typename S::T T;
+  T w[VX];
+#pragma unroll
+  for (int i = 0; i < S::NOPS; ++i) {
+    const unsigned op = S::op(i);
+    if (!(op >> 31)) {
+      pl[op & 15].get(int((op >> 4) & 255) - 128, int((op >> 12) & 15) - 8, w);
+    } else {
+      T& a = acc[(op >> 14) & 7][(op >> 12) & 3];
+      a = fma_t(S::coef(op & 1023), w[(op >> 10) & 3], a);
+    }
+  }
+}
+
+template <class S, int VX, int M, int U, class L>
+__device__ __forceinline__ void run_scatter(const L& pl, typename S::T (&acc)[S::NZ][M][VX]) {
+  typedef typename S::T T;
+  constexpr int NZ = S::NZ;
+  T w[VX];
+#pragma unroll
+  for (int i = 0; i < S::NOPS; ++i) {
+    const unsigned op = S::op(i);
+    if (!(op >> 31)) {
+      pl.get(int((op >> 4) & 255) - 128, int((op >> 12) & 15) - 8, w);
+    } else {
+      const int zi = (op >> 17) & 15;
+      T& a = acc[(U + NZ - zi) % NZ][(op >> 14) & 7][(op >> 12) & 3];
+      a = fma_t(S::coef(op & 1023), w[(op >> 10) & 3], a);
+    }
+  }
+}
+
+// Store a thread tile (rows given by the merge mode) into global memory,
+// masked to the compute box; 128-bit stores when the whole vector is inside.
+template <class T, int VX, int M, bool CM, int BYS>
+__device__ __forceinline__ void store_tile(T* __restrict__ out, const Grid& g, int z, int y0, int x0,
+                                           const T (&acc)[M][VX]) {
+  const bool full_x = (x0 >= g.cx0) && (x0 + VX <= g.cx1) && g.vec_ok;
+#pragma unroll
+  for (int m = 0; m < M; ++m) {
+    const int y = CM ? y0 + m * BYS : y0 + m;
+    if (y < g.cy0 || y >= g.cy1) continue;
+    T* row = out + z * g.sz + y * g.sy;
+    if (full_x) {
+      stg_vec<T, VX>(row + x0, acc[m]);
+    } else {
+#pragma unroll
+      for (int v = 0; v < VX; ++v)
+        if (x0 + v >= g.cx0 && x0 + v < g.cx1) row[x0 + v] = acc[m][v];
+    }
+  }
+}
+
+template <class T, int VX, int M>
+__device__ __forceinline__ void zero_acc(T (&acc)[M][VX]) {
+#pragma unroll
+  for (int m = 0; m < M; ++m)
+#pragma unroll
+    for (int v = 0; v < VX; ++v) acc[m][v] = T(0);
+}
+
+// ===========================================================================
+// OC base / BM / CM with smem = 0: "each GPU thread works on a single output
+// point", or on M merged points. Neighbours are read from global
+// memory through L1 (ld.global.nc). Grid: (x tiles, y tiles, planes).
+// ===========================================================================
+template <class S, int BX, int BY, int M, bool CM>
+__global__ void __launch_bounds__(BX * BY)
+k_naive(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, Grid g) {
+  typedef typename S::T T;
+  constexpr int NROW = CM ? (M - 1) * BY + S::NY : M + S::NY - 1;
+  const int x = g.cx0 + blockIdx.x * BX + threadIdx.x;
+  const int y0 = CM ? g.cy0 + blockIdx.y * BY * M + threadIdx.y
+                    : g.cy0 + (blockIdx.y * BY + threadIdx.y) * M;
+  const int z = g.cz0 + blockIdx.z;
+  if (x >= g.cx1 || y0 >= g.cy1) return;
+  i64 rowoff[NROW];
+#pragma unroll
+  for (int j = 0; j < NROW; ++j) {
+    int y = y0 + j - S::YLO;
+    y = y < g.ny - 1 ? y : g.ny - 1;   // rows past the box only feed masked outputs
+    rowoff[j] = (i64)y * g.sy;
+  }
+  T acc[M][1];
+  zero_acc<T, 1, M>(acc);
+  GlobalPlane<T, 1, NROW> pl[S::NZ];
+#pragma unroll
+  for (int zi = 0; zi < S::NZ; ++zi) pl[zi] = {in + (i64)(z + zi - S::ZLO) * g.sz + x, rowoff, S::YLO};
+  run_gather<S, 1, M>(pl, acc);
+#pragma unroll
+  for (int m = 0; m < M; ++m) {
+    const int y = CM ? y0 + m * BY : y0 + m;
+    if (y < g.cy1) out[(i64)z * g.sz + (i64)y * g.sy + x] = acc[m][0];
+  }
+}
+
+// ===========================================================================
+// Tiled kernel: OC base / BM / CM with smem = 1 (spatial tiling), and
+// TB without ST: an (x,y,z) output tile plus a TT*extent halo is
+// staged once in shared memory (one 3-D TMA box, or cp.async when the rows
+// are not TMA-aligned), then TT time steps are computed in shared memory
+// (ping-pong), each intermediate step on a region shrunk by the extent, with
+// the frame re-imposed; the last step goes to global memory.
+// ===========================================================================
+template <class S, int BX, int BY, int BZ, int VX, int M, bool CM, int TT>
+struct TiledCfg {
+  typedef typename S::T T;
+  static constexpr int ALN = (16 / (int)sizeof(T)) > VX ? (16 / (int)sizeof(T)) : VX;
+  static constexpr int XOFF = ((TT * S::XLO + VX - 1) / VX) * VX;       // smem col of tile x origin
+  static constexpr int LX = ((XOFF + BX + TT * S::XHI + ALN - 1) / ALN) * ALN;
+  static constexpr int LY = BY * M + TT * (S::YLO + S::YHI);
+  static constexpr int LZ = BZ + TT * (S::ZLO + S::ZHI);
+  static constexpr int BUF = ((LX * LY * LZ * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
+  static constexpr int NBUF = TT > 1 ? 2 : 1;
+  static constexpr int SMEM = NBUF * BUF * (int)sizeof(T) + 128;
+  static constexpr int THREADS = (BX / VX) * BY;
+};
+
+template <class S, int BX, int BY, int BZ, int VX, int M, bool CM, int TT, bool TMA>
+__global__ void __launch_bounds__((BX / VX) * BY)
+k_tiled(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, Grid g,
+        const __grid_constant__ TmaDesc tmap) {
+  typedef typename S::T T;
+  typedef TiledCfg<S, BX, BY, BZ, VX, M, CM, TT> C;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  T* buf0 = reinterpret_cast<T*>(smem_raw);
+  T* buf1 = buf0 + C::BUF;
+  unsigned long long* bar = reinterpret_cast<unsigned long long*>(smem_raw + C::NBUF * C::BUF * sizeof(T));
+
+  const int tid = threadIdx.y * (BX / VX) + threadIdx.x;
+  const int xa = (g.cx0 / C::ALN) * C::ALN;            // aligned x origin of the tile grid
+  const int xb = xa + blockIdx.x * BX;
+  const int yb = g.cy0 + blockIdx.y * BY * M;
+  const int zb = g.cz0 + blockIdx.z * BZ;
+  // region origin (array coordinates) of the staged box
+  const int X0 = xb - C::XOFF, Y0 = yb - TT * S::YLO, Z0 = zb - TT * S::ZLO;
+
+  if constexpr (TMA) {
+    if (tid == 0) {
+      tma_prefetch_desc(&tmap);
+      mbar_init(bar, 1);
+      fence_mbar_init();
+    }
+    __syncthreads();
+    if (tid == 0) {
+      mbar_expect_tx(bar, C::LX * C::LY * C::LZ * (unsigned)sizeof(T));
+      tma_load_3d(buf0, &tmap, bar, X0, Y0, Z0);
+    }
+    mbar_wait(bar, 0);
+  } else {
+    const int n = C::LX * C::LY * C::LZ;
+    for (int i = tid; i < n; i += C::THREADS) {
+      const int lx = i % C::LX, ly = (i / C::LX) % C::LY, lz = i / (C::LX * C::LY);
+      const int gx = X0 + lx, gy = Y0 + ly, gz = Z0 + lz;
+      const bool ok = gx >= 0 && gx < g.nx && gy >= 0 && gy < g.ny && gz >= 0 && gz < g.nz;
+      const T* src = ok ? in + (i64)gz * g.sz + (i64)gy * g.sy + gx : in;
+      cp_async_zfill<sizeof(T)>(buf0 + i, src, ok);
+    }
+    cp_async_commit();
+    cp_async_wait<0>();
+    __syncthreads();
+  }
+
+  // intermediate fused steps s = 1 .. TT-1 (temporal blocking)
+  T* src = buf0;
+  T* dst = buf1;
+#pragma unroll 1
+  for (int s = 1; s < TT; ++s) {
+    const int hz0 = (TT - s) * S::ZLO, hz1 = (TT - s) * S::ZHI;
+    const int hy0 = (TT - s) * S::YLO, hy1 = (TT - s) * S::YHI;
+    const int hx0 = (TT - s) * S::XLO, hx1 = (TT - s) * S::XHI;
+    const int RX = BX + hx0 + hx1, RY = BY * M + hy0 + hy1, RZ = BZ + hz0 + hz1;
+    const int n = RX * RY * RZ;
+    for (int i = tid; i < n; i += C::THREADS) {
+      const int rx = i % RX, ry = (i / RX) % RY, rz = i / (RX * RY);
+      const int gx = xb - hx0 + rx, gy = yb - hy0 + ry, gz = zb - hz0 + rz;
+      if (gx < 0 || gx >= g.nx || gy < 0 || gy >= g.ny || gz < 0 || gz >= g.nz) continue;
+      const int li = ((gz - Z0) * C::LY + (gy - Y0)) * C::LX + (gx - X0);
+      const bool upd = gz >= g.uz0 && gz < g.uz1 && gy >= g.uy0 && gy < g.uy1 && gx >= g.ux0 && gx < g.ux1;
+      if (!upd) { dst[li] = src[li]; continue; }
+      T acc = T(0);
+#pragma unroll
+      for (int zi = 0; zi < S::NZ; ++zi)
+#pragma unroll
+        for (int yi = 0; yi < S::NY; ++yi)
+#pragma unroll
+          for (int xi = 0; xi < S::NX; ++xi) {
+            const int id = cidx<S>(zi, yi, xi);
+            if (id >= 0)
+              acc = fma_t(S::coef(id),
+                          src[li + ((zi - S::ZLO) * C::LY + (yi - S::YLO)) * C::LX + (xi - S::XLO)], acc);
+          }
+      dst[li] = acc;
+    }
+    __syncthreads();
+    T* t = src; src = dst; dst = t;
+  }
+
+  // final step: thread tile M x VX per plane, BZ planes
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int row0 = TT * S::YLO + (CM ? ty : ty * M);    // smem row of the first output
+  const int col0 = C::XOFF + tx * VX;
+  const int x0 = xb + tx * VX;
+  const int y0 = yb + (CM ? ty : ty * M);
+#pragma unroll 1
+  for (int zz = 0; zz < BZ; ++zz) {
+    const int z = zb + zz;
+    if (z >= g.cz1) break;
+    T acc[M][VX];
+    zero_acc<T, VX, M>(acc);
+    SmemPlane<T, VX, C::LX> pl[S::NZ];
+#pragma unroll
+    for (int zi = 0; zi < S::NZ; ++zi)
+      pl[zi].p = src + ((TT * S::ZLO + zz + zi - S::ZLO) * C::LY + row0) * C::LX + col0;
+    run_gather<S, VX, M>(pl, acc);
+    store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc);
+  }
+}
+
+// ===========================================================================
+// Streaming kernel: OC ST and its combinations with BM/CM/RT/PR.
+// A CTA owns an (x,y) tile of BX x (BY*M) outputs and a z-chunk of `chunk`
+// output planes (concurrent streaming). Input planes (tile + halo)
+// stream through a ring of shared-memory slots, each staged by one 2-D TMA box
+// (cp.async when rows are not TMA-aligned) signalled on an mbarrier.
+//   RT = false: gather form; the ring holds the NZ planes of the window and
+//               every output plane reads all its slices from shared memory.
+//   RT = true:  retiming: only the newest plane is needed; each value
+//               loaded from it feeds every slice, accumulating into a register
+//               queue of NZ partial-sum sets (one per live output plane).
+//   NS:         planes in flight. NS = 1: the next plane is requested only
+//               after the current one is consumed (no prefetching). NS >= 2:
+//               prefetching: plane p+NS is requested while plane
+//               p+1.. are computed, hiding the per-iteration barrier.
+// ===========================================================================
+template <class S, int BX, int BY, int VX, int M, bool CM, bool RT, int NS>
+struct StreamCfg {
+  typedef typename S::T T;
+  static constexpr int ALN = (16 / (int)sizeof(T)) > VX ? (16 / (int)sizeof(T)) : VX;
+  static constexpr int XOFF = ((S::XLO + VX - 1) / VX) * VX;
+  static constexpr int LX = ((XOFF + BX + S::XHI + ALN - 1) / ALN) * ALN;
+  static constexpr int LY = BY * M + S::YLO + S::YHI;
+  static constexpr int PLANE = ((LX * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
+  static constexpr int NRING = (RT ? 1 : S::NZ) + NS - 1;
+  static constexpr int SMEM = NRING * PLANE * (int)sizeof(T) + 8 * NRING + 128;
+  static constexpr int THREADS = (BX / VX) * BY;
+};
+
+template <class S, int BX, int BY, int VX, int M, bool CM, bool RT, int NS, bool TMA>
+__global__ void __launch_bounds__((BX / VX) * BY)
+k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, Grid g, int chunk,
+         const __grid_constant__ TmaDesc tmap) {
+  typedef typename S::T T;
+  typedef StreamCfg<S, BX, BY, VX, M, CM, RT, NS> C;
+  constexpr int NZ = S::NZ;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  T* ring = reinterpret_cast<T*>(smem_raw);
+  unsigned long long* bar = reinterpret_cast<unsigned long long*>(smem_raw + C::NRING * C::PLANE * sizeof(T));
+
+  const int tid = threadIdx.y * (BX / VX) + threadIdx.x;
+  const int xa = (g.cx0 / C::ALN) * C::ALN;
+  const int xb = xa + blockIdx.x * BX;
+  const int yb = g.cy0 + blockIdx.y * BY * M;
+  const int zs = g.cz0 + blockIdx.z * chunk;
+  const int ze = min(zs + chunk, g.cz1);
+  const int pfirst = zs - S::ZLO;
+  const int nit = (ze - zs) + NZ - 1;                  // planes pfirst .. pfirst+nit-1
+  const int X0 = xb - C::XOFF, Y0 = yb - S::YLO;
+
+  auto issue = [&](int it) {                            // request plane pfirst+it into its slot
+    const int slot = it % C::NRING;
+    T* dst = ring + slot * C::PLANE;
+    if constexpr (TMA) {
+      if (tid == 0) {
+        mbar_expect_tx(&bar[slot], C::LX * C::LY * (unsigned)sizeof(T));
+        tma_load_3d(dst, &tmap, &bar[slot], X0, Y0, pfirst + it);
+      }
+    } else {
+      const int gz = pfirst + it;
+      const T* plane = in + (i64)gz * g.sz;
+      for (int i = tid; i < C::LX * C::LY; i += C::THREADS) {
+        const int lx = i % C::LX, ly = i / C::LX;
+        const int gx = X0 + lx, gy = Y0 + ly;
+        const bool ok = gx >= 0 && gx < g.nx && gy >= 0 && gy < g.ny;
+        cp_async_zfill<sizeof(T)>(dst + i, ok ? plane + (i64)gy * g.sy + gx : in, ok);
+      }
+    }
+  };
+  auto wait_plane = [&](int it) {
+    if constexpr (TMA) {
+      mbar_wait(&bar[it % C::NRING], (unsigned)((it / C::NRING) & 1));
+    } else {
+      cp_async_wait<NS - 1>();
+      __syncthreads();
+    }
+  };
+
+  if constexpr (TMA) {
+    if (tid == 0) {
+      tma_prefetch_desc(&tmap);
+      for (int s = 0; s < C::NRING; ++s) mbar_init(&bar[s], 1);
+      fence_mbar_init();
+    }
+    __syncthreads();
+  }
+  // prologue: planes 0 .. NS-2 in flight. Plane it+NS-1 goes to the slot of
+  // plane it-W (W = window: NZ for gather, 1 for RT), last read in iteration
+  // it-1 and released by that iteration's closing barrier.
+#pragma unroll 1
+  for (int it = 0; it < NS - 1; ++it) {
+    if (it < nit) issue(it);
+    if constexpr (!TMA) cp_async_commit();
+  }
+
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int row0 = S::YLO + (CM ? ty : ty * M);
+  const int col0 = C::XOFF + tx * VX;
+  const int x0 = xb + tx * VX;
+  const int y0 = yb + (CM ? ty : ty * M);
+
+  if constexpr (RT) {
+    T acc[NZ][M][VX];
+#pragma unroll
+    for (int q = 0; q < NZ; ++q) zero_acc<T, VX, M>(acc[q]);
+#pragma unroll 1
+    for (int itb = 0; itb < nit; itb += NZ) {
+      // unrolled by NZ so that the register-queue rotation is compile-time
+      static_for<0, NZ>([&](auto ic) {
+        constexpr int U = decltype(ic)::value;
+        const int it = itb + U;
+        if (it < nit) {
+          if (it + NS - 1 < nit) issue(it + NS - 1);
+          if constexpr (!TMA) cp_async_commit();
+          wait_plane(it);
+          zero_acc<T, VX, M>(acc[U]);                    // output plane pfirst+it+ZLO starts
+          SmemPlane<T, VX, C::LX> pl{ring + (it % C::NRING) * C::PLANE + row0 * C::LX + col0};
+          run_scatter<S, VX, M, U>(pl, acc);
+          const int z = pfirst + it - S::ZHI;             // output completed by this plane
+          if (z >= zs) store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc[(U + 1) % NZ]);
+          __syncthreads();                                // slot it%NRING may be refilled
+        }
+      });
+    }
+  } else {
+#pragma unroll 1
+    for (int it = 0; it < nit; ++it) {
+      if (it + NS - 1 < nit) issue(it + NS - 1);
+      if constexpr (!TMA) cp_async_commit();
+      wait_plane(it);
+      if (it >= NZ - 1) {
+        const int z = pfirst + it - S::ZHI;
+        T acc[M][VX];
+        zero_acc<T, VX, M>(acc);
+        SmemPlane<T, VX, C::LX> pl[NZ];
+#pragma unroll
+        for (int zi = 0; zi < NZ; ++zi)                  // plane z + zi - ZLO
+          pl[zi].p = ring + ((it - (NZ - 1) + zi) % C::NRING) * C::PLANE + row0 * C::LX + col0;
+        run_gather<S, VX, M>(pl, acc);
+        store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc);
+      }
+      __syncthreads();                                    // oldest slot may be refilled
+    }
+  }
+}
+
+}  // namespace smart

@@ -1,0 +1,127 @@
+// aot_kernels.cu -- pattern-independent kernels compiled ahead of time (nvcc,
+// sm_100a): the frame copy of the ping-pong setup and the
+// device side of the counter-based input generator (reading C-3).
+#include "internal.h"
+
+namespace smart_rt {
+
+namespace {
+
+// Frame = points outside the update box. Three disjoint groups are
+// enumerated so only frame points are touched:
+//   A: whole planes z < uz0 or z >= uz1
+//   B: planes uz0..uz1-1, whole rows y < uy0 or y >= uy1
+//   C: planes uz0..uz1-1, rows uy0..uy1-1, columns x < ux0 or x >= ux1
+template <class W>
+__global__ void k_frame_copy(const W* __restrict__ src, W* __restrict__ dst, GridArg g) {
+  const long long nzA = (long long)g.uz0 + (g.nz - g.uz1);
+  const long long nyB = (long long)g.uy0 + (g.ny - g.uy1);
+  const long long nxC = (long long)g.ux0 + (g.nx - g.ux1);
+  const long long midz = g.uz1 - g.uz0, midy = g.uy1 - g.uy0;
+  const long long nA = nzA * g.ny * g.nx;
+  const long long nB = midz * nyB * g.nx;
+  const long long nC = midz * midy * nxC;
+  const long long total = nA + nB + nC;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
+       i += (long long)gridDim.x * blockDim.x) {
+    long long z, y, x;
+    if (i < nA) {
+      x = i % g.nx;
+      y = (i / g.nx) % g.ny;
+      long long zz = i / ((long long)g.nx * g.ny);
+      z = zz < g.uz0 ? zz : g.uz1 + (zz - g.uz0);
+    } else if (i < nA + nB) {
+      long long k = i - nA;
+      x = k % g.nx;
+      long long yy = (k / g.nx) % nyB;
+      z = g.uz0 + k / ((long long)g.nx * nyB);
+      y = yy < g.uy0 ? yy : g.uy1 + (yy - g.uy0);
+    } else {
+      long long k = i - nA - nB;
+      long long xx = k % nxC;
+      y = g.uy0 + (k / nxC) % midy;
+      z = g.uz0 + k / (nxC * midy);
+      x = xx < g.ux0 ? xx : g.ux1 + (xx - g.ux0);
+    }
+    const long long p = z * g.sz + y * g.sy + x;
+    dst[p] = src[p];
+  }
+}
+
+__device__ __forceinline__ unsigned long long mix64(unsigned long long x) {
+  unsigned long long z = x + 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+template <class T>
+__device__ __forceinline__ T value_of(unsigned long long h, int kind);
+
+template <>
+__device__ __forceinline__ double value_of<double>(unsigned long long h, int kind) {
+  if (kind == 0) return __longlong_as_double((long long)((h >> 12) | 0x3FF0000000000000ull));
+  return (double)((long long)((h >> 53) % 2047ull) - 1023);
+}
+template <>
+__device__ __forceinline__ float value_of<float>(unsigned long long h, int kind) {
+  if (kind == 0) return __uint_as_float((unsigned)((h >> 41) | 0x3F800000ull));
+  return (float)((long long)((h >> 53) % 2047ull) - 1023);
+}
+
+template <class T>
+__global__ void k_fill(T* __restrict__ dst, long long bz, long long by, long long bx, long long oz,
+                       long long oy, long long ox, long long gy, long long gx, unsigned long long key,
+                       int kind) {
+  const long long total = bz * by * bx;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
+       i += (long long)gridDim.x * blockDim.x) {
+    const long long x = i % bx, y = (i / bx) % by, z = i / (bx * by);
+    const unsigned long long gidx =
+        (unsigned long long)(((oz + z) * gy + (oy + y)) * gx + (ox + x));
+    dst[i] = value_of<T>(mix64(gidx ^ key), kind);
+  }
+}
+
+int grid_for(long long n) {
+  long long b = (n + 255) / 256;
+  const long long cap = 148LL * 16;
+  if (b > cap) b = cap;
+  if (b < 1) b = 1;
+  return (int)b;
+}
+
+}  // namespace
+
+int launch_frame_copy(const void* src, void* dst, int elem, const GridArg& g, cudaStream_t s) {
+  const long long vol = (long long)g.nz * g.ny * g.nx;
+  const long long inner = (long long)(g.uz1 - g.uz0) * (g.uy1 - g.uy0) * (g.ux1 - g.ux0);
+  const long long n = vol - inner;
+  if (n <= 0) return STENCIL_OK;
+  if (elem == 8)
+    k_frame_copy<unsigned long long><<<grid_for(n), 256, 0, s>>>(
+        (const unsigned long long*)src, (unsigned long long*)dst, g);
+  else
+    k_frame_copy<unsigned><<<grid_for(n), 256, 0, s>>>((const unsigned*)src, (unsigned*)dst, g);
+  g_launches.fetch_add(1);
+  SM_CUDA(cudaGetLastError());
+  return STENCIL_OK;
+}
+
+int launch_fill(void* dst, int dtype, const int64_t box[3], const int64_t org[3], const int64_t gdim[3],
+                uint64_t seed, int kind, cudaStream_t s) {
+  const long long n = box[0] * box[1] * box[2];
+  if (n <= 0) return STENCIL_OK;
+  const unsigned long long key = (unsigned long long)seed * 0xD1B54A32D192ED03ull;
+  if (dtype == STENCIL_F64)
+    k_fill<double><<<grid_for(n), 256, 0, s>>>((double*)dst, box[0], box[1], box[2], org[0], org[1],
+                                                org[2], gdim[1], gdim[2], key, kind);
+  else
+    k_fill<float><<<grid_for(n), 256, 0, s>>>((float*)dst, box[0], box[1], box[2], org[0], org[1],
+                                               org[2], gdim[1], gdim[2], key, kind);
+  g_launches.fetch_add(1);
+  SM_CUDA(cudaGetLastError());
+  return STENCIL_OK;
+}
+
+}  // namespace smart_rt

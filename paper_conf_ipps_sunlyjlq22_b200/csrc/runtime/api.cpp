@@ -1,0 +1,701 @@
+// api.cpp -- the C ABI of include/stencil.h: validation, pattern ingestion,
+// OC lattice, parameter settings, launch configuration and the time loop.
+// SURVEY §8(a) rows a1 (pattern ingestion), a2 (OC validation + settings),
+// a4 (frame / ping-pong setup), a5 (dispatch to the OC kernel family) and a6
+// (time loop). Citations: PAPER.md line numbers (P:L<n>).
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+
+#include "internal.h"
+
+namespace smart_rt {
+
+std::atomic<uint64_t> g_launches{0};
+
+// ----------------------------------------------------------------- errors
+static thread_local std::string t_err;
+
+void set_error(const char* fmt, ...) {
+  char buf[4096];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  t_err = buf;
+}
+void clear_error() { t_err.clear(); }
+
+// ------------------------------------------------------------- driver API
+static Driver g_drv;
+static int g_drv_state = 0;   // 0 unknown, 1 ok, -1 failed
+static std::mutex g_drv_mu;
+
+template <class F>
+static bool entry(const char* name, F* fp) {
+  void* p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q) != cudaSuccess || q != cudaDriverEntryPointSuccess ||
+      !p)
+    return false;
+  *fp = reinterpret_cast<F>(p);
+  return true;
+}
+
+int get_driver(const Driver** out) {
+  std::lock_guard<std::mutex> lk(g_drv_mu);
+  if (g_drv_state == 0) {
+    bool ok = entry("cuModuleLoadData", &g_drv.moduleLoadData) && entry("cuModuleUnload", &g_drv.moduleUnload) &&
+              entry("cuModuleGetFunction", &g_drv.moduleGetFunction) &&
+              entry("cuFuncSetAttribute", &g_drv.funcSetAttribute) &&
+              entry("cuFuncGetAttribute", &g_drv.funcGetAttribute) && entry("cuLaunchKernel", &g_drv.launchKernel) &&
+              entry("cuTensorMapEncodeTiled", &g_drv.tensorMapEncodeTiled) &&
+              entry("cuGetErrorString", &g_drv.getErrorString);
+    g_drv_state = ok ? 1 : -1;
+  }
+  if (g_drv_state != 1) SM_FAIL(STENCIL_E_CUDA, "CUDA driver entry points unavailable (no GPU driver?)");
+  *out = &g_drv;
+  return STENCIL_OK;
+}
+
+const char* cu_errstr(CUresult r) {
+  const char* s = nullptr;
+  if (g_drv_state == 1 && g_drv.getErrorString) g_drv.getErrorString(r, &s);
+  return s ? s : "unknown CUDA driver error";
+}
+
+// ------------------------------------------------------------ OC lattice
+// Table I: BM xor CM; RT => ST; PR => ST.
+static bool oc_valid(uint32_t oc) {
+  if (oc >= 64) return false;
+  const bool st = oc & STENCIL_OC_ST, bm = oc & STENCIL_OC_BM, cm = oc & STENCIL_OC_CM;
+  const bool rt = oc & STENCIL_OC_RT, pr = oc & STENCIL_OC_PR;
+  if (bm && cm) return false;
+  if ((rt || pr) && !st) return false;
+  return true;
+}
+
+static const char* oc_name_static(uint32_t oc) {
+  static std::string names[64];
+  static std::once_flag once;
+  std::call_once(once, [] {
+    const char* ab[6] = {"ST", "TB", "BM", "CM", "RT", "PR"};
+    const uint32_t bit[6] = {STENCIL_OC_ST, STENCIL_OC_TB, STENCIL_OC_BM, STENCIL_OC_CM, STENCIL_OC_RT, STENCIL_OC_PR};
+    for (uint32_t m = 0; m < 64; ++m) {
+      std::string s;
+      for (int k = 0; k < 6; ++k)
+        if (m & bit[k]) s += (s.empty() ? "" : "_") + std::string(ab[k]);
+      names[m] = s.empty() ? "base" : s;
+    }
+  });
+  if (!oc_valid(oc)) return nullptr;
+  return names[oc].c_str();
+}
+
+// ------------------------------------------------------ parameter space
+static bool pow2(int v) { return v > 0 && (v & (v - 1)) == 0; }
+
+static int family_of(uint32_t oc, int smem) {
+  const bool st = oc & STENCIL_OC_ST, tb = oc & STENCIL_OC_TB;
+  if (st) return tb ? FAM_STREAM_TB : FAM_STREAM;
+  if (tb) return FAM_TILED;
+  return smem ? FAM_TILED : FAM_NAIVE;
+}
+
+// Defaults (k = 0 setting) per OC and dtype.
+static void default_params(uint32_t oc, int ndim, int dtype, stencil_params_t* p) {
+  const int vmax = dtype == STENCIL_F64 ? 2 : 4;
+  const bool merge = oc & (STENCIL_OC_BM | STENCIL_OC_CM);
+  memset(p, 0, sizeof *p);
+  p->smem = 0;
+  p->merge = merge ? 2 : 1;
+  p->tb_steps = (oc & STENCIL_OC_TB) ? 2 : 1;
+  p->pr_stages = (oc & STENCIL_OC_PR) ? 2 : 1;
+  p->stream_chunk = 0;   // auto
+  const int fam = family_of(oc, 0);
+  if (fam == FAM_NAIVE) {
+    p->bx = 32; p->by = merge ? 4 : 8; p->bz = 1; p->vx = 1;
+  } else if (fam == FAM_TILED) {
+    p->vx = vmax; p->bx = 16 * vmax; p->by = merge ? 4 : 8; p->bz = (oc & STENCIL_OC_TB) ? 4 : 8;
+    if (ndim == 2) p->bz = 1;
+  } else {
+    p->vx = vmax; p->bx = 32 * vmax; p->by = merge ? 4 : 8; p->bz = 1;
+  }
+}
+
+// counter-based hash for the seeded settings sampler
+static uint64_t mix64(uint64_t x) {
+  uint64_t z = x + 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+template <size_t N>
+static int pick(uint64_t& h, const int (&choices)[N]) {
+  h = mix64(h);
+  return choices[h % N];
+}
+
+static void sample_params(uint32_t oc, int ndim, int dtype, uint64_t seed, int k, stencil_params_t* p) {
+  default_params(oc, ndim, dtype, p);
+  if (k <= 0) return;
+  uint64_t h = mix64(seed ^ ((uint64_t)oc << 32) ^ (uint64_t)k * 0x632BE59BD9B4E019ull);
+  const bool merge = oc & (STENCIL_OC_BM | STENCIL_OC_CM);
+  const bool st = oc & STENCIL_OC_ST, tb = oc & STENCIL_OC_TB;
+  if (!st && !tb) { const int s[] = {0, 1}; p->smem = pick(h, s); }
+  if (merge) { const int s[] = {2, 4, 8}; p->merge = pick(h, s); }
+  if (tb) { const int s[] = {2, 4}; p->tb_steps = pick(h, s); }
+  if (oc & STENCIL_OC_PR) { const int s[] = {2, 4}; p->pr_stages = pick(h, s); }
+  const int fam = family_of(oc, p->smem);
+  if (fam == FAM_NAIVE) {
+    const int sx[] = {32, 64, 128}, sy[] = {1, 2, 4, 8};
+    p->bx = pick(h, sx); p->by = pick(h, sy); p->vx = 1;
+  } else {
+    const int vmax = dtype == STENCIL_F64 ? 2 : 4;
+    const int sv[] = {1, 2, 4};
+    p->vx = std::min(pick(h, sv), vmax);
+    const int sx[] = {16, 32, 64, 128};
+    p->bx = std::max(pick(h, sx) * p->vx / (p->vx > 2 ? 2 : 1), 8 * p->vx);
+    const int sy[] = {2, 4, 8, 16};
+    p->by = pick(h, sy);
+    if (fam == FAM_TILED) { const int sz[] = {2, 4, 8}; p->bz = ndim == 2 ? 1 : pick(h, sz); }
+    if (st) { const int sc[] = {0, 32, 64, 128, 256}; p->stream_chunk = pick(h, sc); }
+  }
+  // keep the CTA within 32..1024 threads
+  while ((p->bx / std::max(p->vx, 1)) * p->by > 1024 && p->by > 1) p->by /= 2;
+  while ((p->bx / std::max(p->vx, 1)) * p->by < 32) p->by *= 2;
+}
+
+// ------------------------------------------------------------- pattern
+static int build_pattern(stencil_plan_s* P) {
+  const int r = P->order, w = 2 * r + 1;
+  const bool two = P->ndim == 2;
+  const int tsize = two ? w * w : w * w * w;
+  P->pat = Pattern();
+  Pattern& pat = P->pat;
+  int zlo = 0, zhi = 0, ylo = 0, yhi = 0, xlo = 0, xhi = 0;
+  for (int t = 0; t < tsize; ++t) {
+    if (!P->access[t]) continue;
+    int a, b, c;   // slowest..fastest offsets of the user tensor
+    if (two) { a = 0; b = t / w - r; c = t % w - r; }
+    else { a = t / (w * w) - r; b = (t / w) % w - r; c = t % w - r; }
+    pat.dz.push_back(a); pat.dy.push_back(b); pat.dx.push_back(c);
+    pat.c.push_back(P->coeffs[t]);
+    zlo = std::max(zlo, -a); zhi = std::max(zhi, a);
+    ylo = std::max(ylo, -b); yhi = std::max(yhi, b);
+    xlo = std::max(xlo, -c); xhi = std::max(xhi, c);
+  }
+  pat.nnz = (int)pat.c.size();
+  pat.zlo = zlo; pat.zhi = zhi; pat.ylo = ylo; pat.yhi = yhi; pat.xlo = xlo; pat.xhi = xhi;
+  return STENCIL_OK;
+}
+
+// The 3-D kernel view of the grid. 3-D: identity. 2-D [ny][nx]: non-streaming
+// families see [1][ny][nx]; streaming families stream along y and see
+// [ny][1][nx] (the streaming dimension is the slowest one, C-13).
+static void build_view(stencil_plan_s* P, int fam) {
+  const int r = P->order;
+  if (P->ndim == 3) {
+    for (int k = 0; k < 3; ++k) { P->vdims[k] = P->dims[k]; P->frame[k] = r; }
+    return;
+  }
+  const bool stream = fam == FAM_STREAM || fam == FAM_STREAM_TB;
+  Pattern& pat = P->pat;
+  if (stream) {
+    P->vdims[0] = P->dims[0]; P->vdims[1] = 1; P->vdims[2] = P->dims[1];
+    P->frame[0] = r; P->frame[1] = 0; P->frame[2] = r;
+    // (0, dy, dx) -> (dy, 0, dx)
+    for (int i = 0; i < pat.nnz; ++i) { pat.dz[i] = pat.dy[i]; pat.dy[i] = 0; }
+    pat.zlo = pat.ylo; pat.zhi = pat.yhi; pat.ylo = pat.yhi = 0;
+  } else {
+    P->vdims[0] = 1; P->vdims[1] = P->dims[0]; P->vdims[2] = P->dims[1];
+    P->frame[0] = 0; P->frame[1] = r; P->frame[2] = r;
+  }
+}
+
+// ---------------------------------------------------- variant + feasibility
+struct TmaBox { int lx, ly, lz; };
+
+static TmaBox tma_box(const Variant& v, const Pattern& p, int elem) {
+  const int aln = std::max(16 / elem, v.vx);
+  auto ru = [](int a, int b) { return (a + b - 1) / b * b; };
+  if (v.family == FAM_TILED) {
+    const int xoff = ru(v.tt * p.xlo, v.vx);
+    return {ru(xoff + v.bx + v.tt * p.xhi, aln), v.by * v.m + v.tt * (p.ylo + p.yhi),
+            v.bz + v.tt * (p.zlo + p.zhi)};
+  }
+  const int xoff = ru(p.xlo, v.vx);
+  return {ru(xoff + v.bx + p.xhi, aln), v.by * v.m + p.ylo + p.yhi, 1};
+}
+
+static int resolve_variant(stencil_plan_s* P) {
+  const stencil_params_t& p = P->params;
+  const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+  const int fam = family_of(P->oc, p.smem);
+  Variant v;
+  v.family = fam;
+  v.bx = p.bx; v.by = p.by; v.bz = p.bz; v.vx = p.vx; v.m = p.merge;
+  v.cm = (P->oc & STENCIL_OC_CM) != 0;
+  v.tt = (P->oc & STENCIL_OC_TB) ? p.tb_steps : 1;
+  v.rt = (P->oc & STENCIL_OC_RT) != 0;
+  v.ns = (P->oc & STENCIL_OC_PR) ? p.pr_stages : 1;
+  if (fam == FAM_NAIVE) { v.vx = 1; v.bz = 1; }
+  if (fam == FAM_STREAM || fam == FAM_STREAM_TB) v.bz = 1;
+  if (P->ndim == 2) {
+    if (fam == FAM_STREAM || fam == FAM_STREAM_TB) { v.by = 1; v.m = 1; }
+    else v.bz = 1;
+  }
+  if (fam == FAM_STREAM_TB)
+    SM_FAIL(STENCIL_E_OC_INFEASIBLE, "OC %s: streaming + temporal blocking kernel not built yet",
+            oc_name_static(P->oc));
+  if (v.vx != 1 && v.vx != 2 && v.vx != 4) SM_FAIL(STENCIL_E_INVAL, "vx must be 1, 2 or 4");
+  if (v.vx * elem > 32) SM_FAIL(STENCIL_E_INVAL, "vx*sizeof(T) must be <= 32 bytes");
+  if (!pow2(v.bx) || !pow2(v.by) || !pow2(v.bz) || !pow2(v.m) || v.bx < v.vx)
+    SM_FAIL(STENCIL_E_INVAL, "tile parameters must be powers of two (bx=%d by=%d bz=%d merge=%d vx=%d)", v.bx,
+            v.by, v.bz, v.m, v.vx);
+  if (v.m > 8) SM_FAIL(STENCIL_E_INVAL, "merge factor must be <= 8");
+  if (v.tt < 1 || v.tt > 8) SM_FAIL(STENCIL_E_INVAL, "tb_steps must be in 1..8");
+  if (v.ns < 1 || v.ns > 4) SM_FAIL(STENCIL_E_INVAL, "pr_stages must be in 1..4");
+  const int thr = v.threads();
+  if (thr < 32 || thr > 1024)
+    SM_FAIL(STENCIL_E_OC_INFEASIBLE, "CTA of %d threads outside 32..1024", thr);
+  const int smem = v.smem_bytes(P->pat, elem);
+  if (smem > 232448)
+    SM_FAIL(STENCIL_E_OC_INFEASIBLE, "OC %s needs %d B of shared memory per CTA (> 227 KB)",
+            oc_name_static(P->oc), smem);
+  // TMA staging when rows are 16-byte multiples and the box fits 256^3
+  v.tma = false;
+  if (fam == FAM_TILED || fam == FAM_STREAM) {
+    const TmaBox b = tma_box(v, P->pat, elem);
+    const bool rows_ok = (P->vdims[2] * elem) % 16 == 0;
+    v.tma = rows_ok && b.lx <= 256 && b.ly <= 256 && b.lz <= 256 && getenv("STENCIL_NO_TMA") == nullptr;
+  }
+  v.chunk = p.stream_chunk;
+  P->var = v;
+  return STENCIL_OK;
+}
+
+static int validate_params(const stencil_params_t* p) {
+  for (int k = 0; k < 3; ++k)
+    if (p->reserved[k] != 0) SM_FAIL(STENCIL_E_INVAL, "stencil_params_t.reserved must be 0");
+  if (p->smem < -1 || p->smem > 1) SM_FAIL(STENCIL_E_INVAL, "smem must be -1, 0 or 1");
+  const int32_t* f = &p->bx;
+  for (int k = 0; k < 8; ++k)
+    if (f[k] < 0) SM_FAIL(STENCIL_E_INVAL, "negative parameter");
+  return STENCIL_OK;
+}
+
+static void merge_params(const stencil_params_t* user, stencil_params_t* out) {
+  if (!user) return;
+  if (user->smem >= 0) out->smem = user->smem;
+  if (user->bx) out->bx = user->bx;
+  if (user->by) out->by = user->by;
+  if (user->bz) out->bz = user->bz;
+  if (user->vx) out->vx = user->vx;
+  if (user->merge) out->merge = user->merge;
+  if (user->stream_chunk) out->stream_chunk = user->stream_chunk;
+  if (user->tb_steps) out->tb_steps = user->tb_steps;
+  if (user->pr_stages) out->pr_stages = user->pr_stages;
+}
+
+// ------------------------------------------------------------ grid args
+static GridArg make_grid(const stencil_plan_s* P, int elem_vx) {
+  GridArg g{};
+  g.nz = (int)P->vdims[0]; g.ny = (int)P->vdims[1]; g.nx = (int)P->vdims[2];
+  g.sy = P->vdims[2];
+  g.sz = P->vdims[1] * P->vdims[2];
+  g.uz0 = P->frame[0]; g.uz1 = g.nz - P->frame[0];
+  g.uy0 = P->frame[1]; g.uy1 = g.ny - P->frame[1];
+  g.ux0 = P->frame[2]; g.ux1 = g.nx - P->frame[2];
+  g.cz0 = g.uz0; g.cz1 = g.uz1; g.cy0 = g.uy0; g.cy1 = g.uy1; g.cx0 = g.ux0; g.cx1 = g.ux1;
+  g.vec_ok = (g.nx % elem_vx) == 0;
+  return g;
+}
+
+static int ensure_loaded(stencil_plan_s* P) {
+  if (P->loaded) return STENCIL_OK;
+  const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+  if (P->cubin.empty()) SM_TRY(compile_variant(P->pat, P->dtype, P->var, &P->lowered, &P->cubin));
+  SM_TRY(load_kernel(P->src, P->cubin, P->lowered, P->var.smem_bytes(P->pat, elem), &P->kern));
+  P->loaded = true;
+  return STENCIL_OK;
+}
+
+static int get_tmap(stencil_plan_s* P, const Variant& v, const void* buf, CUtensorMap** out) {
+  auto it = P->tmaps.find(buf);
+  if (it != P->tmaps.end() && v.family == P->var.family && v.tt == P->var.tt) {
+    *out = &it->second;
+    return STENCIL_OK;
+  }
+  const Driver* d = nullptr;
+  SM_TRY(get_driver(&d));
+  const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+  if (((uintptr_t)buf) % 16) SM_FAIL(STENCIL_E_INVAL, "TMA staging needs 16-byte aligned grid pointers");
+  const TmaBox b = tma_box(v, P->pat, elem);
+  CUtensorMap m;
+  cuuint64_t gdim[3] = {(cuuint64_t)P->vdims[2], (cuuint64_t)P->vdims[1], (cuuint64_t)P->vdims[0]};
+  cuuint64_t gstr[2] = {(cuuint64_t)(P->vdims[2] * elem), (cuuint64_t)(P->vdims[2] * P->vdims[1] * elem)};
+  cuuint32_t box[3] = {(cuuint32_t)b.lx, (cuuint32_t)b.ly, (cuuint32_t)b.lz};
+  cuuint32_t es[3] = {1, 1, 1};
+  CUresult r = d->tensorMapEncodeTiled(&m, elem == 8 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                                       3, const_cast<void*>(buf), gdim, gstr, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                       CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) SM_FAIL(STENCIL_E_CUDA, "cuTensorMapEncodeTiled: %s", cu_errstr(r));
+  if (v.family == P->var.family && v.tt == P->var.tt) {
+    P->tmaps[buf] = m;
+    *out = &P->tmaps[buf];
+  } else {
+    static thread_local CUtensorMap tmp;
+    tmp = m;
+    *out = &tmp;
+  }
+  return STENCIL_OK;
+}
+
+static int auto_chunk(const stencil_plan_s* P, const Variant& v, int czlen, long long tiles_xy) {
+  if (v.chunk > 0) return std::min(v.chunk, czlen);
+  // enough CTAs for ~8 per SM, but chunks of at least 16 planes (halo reuse)
+  long long target = 148LL * 8;
+  int c = 1;
+  while (c < czlen && tiles_xy * ((czlen + c - 1) / c) > target) c *= 2;
+  (void)P;
+  return std::max(std::min(c, czlen), std::min(16, czlen));
+}
+
+// Launch the main variant (or `k` for a TB remainder) for one application of
+// the kernel: src -> dst over the compute box of g.
+static int launch_sweep(stencil_plan_s* P, const Variant& v, const Kernel& k, const void* src, void* dst,
+                        const GridArg& g) {
+  const Driver* d = nullptr;
+  SM_TRY(get_driver(&d));
+  const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+  const int czlen = g.cz1 - g.cz0, cylen = g.cy1 - g.cy0, cxlen = g.cx1 - g.cx0;
+  if (czlen <= 0 || cylen <= 0 || cxlen <= 0) return STENCIL_OK;
+  const int aln = std::max(16 / elem, v.vx);
+  unsigned gx, gy, gz, bx, by;
+  int chunk = 0;
+  CUtensorMap* tm = nullptr;
+  CUtensorMap dummy;
+  memset(&dummy, 0, sizeof dummy);
+  void* args[5];
+  const void* in = src;
+  void* out = dst;
+  GridArg gg = g;
+  args[0] = (void*)&in;
+  args[1] = (void*)&out;
+  args[2] = (void*)&gg;
+  int nargs = 3;
+  if (v.family == FAM_NAIVE) {
+    gx = (cxlen + v.bx - 1) / v.bx;
+    gy = (cylen + v.by * v.m - 1) / (v.by * v.m);
+    gz = czlen;
+    bx = v.bx; by = v.by;
+  } else {
+    const int xa = (g.cx0 / aln) * aln;
+    gx = (g.cx1 - xa + v.bx - 1) / v.bx;
+    gy = (cylen + v.by * v.m - 1) / (v.by * v.m);
+    bx = v.bx / v.vx; by = v.by;
+    if (v.tma) SM_TRY(get_tmap(P, v, src, &tm));
+    if (v.family == FAM_TILED) {
+      gz = (czlen + v.bz - 1) / v.bz;
+      args[3] = tm ? (void*)tm : (void*)&dummy;
+      nargs = 4;
+    } else {
+      chunk = auto_chunk(P, v, czlen, (long long)gx * gy);
+      gz = (czlen + chunk - 1) / chunk;
+      args[3] = (void*)&chunk;
+      args[4] = tm ? (void*)tm : (void*)&dummy;
+      nargs = 5;
+    }
+  }
+  (void)nargs;
+  if (gy > 65535 || gz > 65535) SM_FAIL(STENCIL_E_OC_INFEASIBLE, "grid too large for this tile setting");
+  const int smem = v.smem_bytes(P->pat, elem);
+  CUresult r = d->launchKernel(k.fn, gx, gy, gz, bx, by, 1, smem, (CUstream)P->stream, args, nullptr);
+  g_launches.fetch_add(1);
+  if (r != CUDA_SUCCESS) SM_FAIL(STENCIL_E_CUDA, "cuLaunchKernel(%s): %s", P->lowered.c_str(), cu_errstr(r));
+  return STENCIL_OK;
+}
+
+static int get_tb_rem_kernel(stencil_plan_s* P, int tt, Variant* vout, Kernel* kout) {
+  Variant v = P->var;
+  v.tt = tt;
+  const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+  if (v.family == FAM_TILED && v.tma) {
+    const TmaBox b = tma_box(v, P->pat, elem);
+    v.tma = b.lx <= 256 && b.ly <= 256 && b.lz <= 256;
+  }
+  *vout = v;
+  auto it = P->tb_rem.find(tt);
+  if (it != P->tb_rem.end()) { *kout = it->second; return STENCIL_OK; }
+  std::string low;
+  std::vector<char> bin;
+  SM_TRY(compile_variant(P->pat, P->dtype, v, &low, &bin));
+  Kernel k;
+  SM_TRY(load_kernel(generate_source(P->pat, P->dtype, v), bin, low, v.smem_bytes(P->pat, elem), &k));
+  P->tb_rem[tt] = k;
+  *kout = k;
+  return STENCIL_OK;
+}
+
+int run_device(stencil_plan_s* P, const void* in, void* out, int steps);
+
+}  // namespace smart_rt
+
+using namespace smart_rt;
+
+stencil_plan_s::~stencil_plan_s() {
+  if (h_in_dev) cudaFree(h_in_dev);
+  if (h_out_dev) cudaFree(h_out_dev);
+  if (h_ws_dev) cudaFree(h_ws_dev);
+  if (comm) comm_destroy(comm);
+}
+
+namespace smart_rt {
+
+int run_device(stencil_plan_s* P, const void* in, void* out, int steps) {
+  const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+  const size_t bytes = (size_t)P->vdims[0] * P->vdims[1] * P->vdims[2] * elem;
+  if (!in || !out) SM_FAIL(STENCIL_E_INVAL, "null grid pointer");
+  if (in == out) SM_FAIL(STENCIL_E_INVAL, "in and out must be distinct buffers");
+  if (steps < 0) SM_FAIL(STENCIL_E_INVAL, "steps must be >= 0");
+  if ((uintptr_t)in % 16 || (uintptr_t)out % 16) SM_FAIL(STENCIL_E_INVAL, "grid pointers must be 16-byte aligned");
+  if (steps == 0) {
+    SM_CUDA(cudaMemcpyAsync(out, in, bytes, cudaMemcpyDeviceToDevice, P->stream));
+    return STENCIL_OK;
+  }
+  const int T = P->var.family == FAM_TILED || P->var.family == FAM_STREAM_TB ? P->var.tt : 1;
+  const int launches = (steps + T - 1) / T;
+  if (launches >= 2 && (!P->ws || P->ws_bytes < bytes))
+    SM_FAIL(STENCIL_E_STATE, "steps=%d needs a workspace of %zu bytes (stencil_plan_set_workspace)", steps, bytes);
+  SM_TRY(ensure_loaded(P));
+  const GridArg g = make_grid(P, P->var.vx);
+  // a4: frame of the input into every buffer the sweep writes (fixed thereafter)
+  SM_TRY(launch_frame_copy(in, out, elem, g, P->stream));
+  if (launches >= 2) SM_TRY(launch_frame_copy(in, P->ws, elem, g, P->stream));
+  const void* src = in;
+  for (int i = 0; i < launches; ++i) {
+    void* dst = ((launches - 1 - i) % 2 == 0) ? out : P->ws;
+    const int tt = std::min(T, steps - i * T);
+    if (tt == T) {
+      SM_TRY(launch_sweep(P, P->var, P->kern, src, dst, g));
+    } else {
+      Variant v;
+      Kernel k;
+      SM_TRY(get_tb_rem_kernel(P, tt, &v, &k));
+      SM_TRY(launch_sweep(P, v, k, src, dst, g));
+    }
+    src = dst;
+  }
+  SM_CUDA(cudaGetLastError());
+  return STENCIL_OK;
+}
+
+}  // namespace smart_rt
+
+// =====================================================================
+// C ABI
+// =====================================================================
+extern "C" {
+
+const char* stencil_last_error(void) { return t_err.c_str(); }
+uint64_t stencil_launch_count(void) { return g_launches.load(); }
+int stencil_abi_version(void) { return STENCIL_ABI_VERSION; }
+
+int stencil_oc_valid(uint32_t oc) { return oc_valid(oc) ? 1 : 0; }
+
+int stencil_oc_list(uint32_t* ids) {
+  int n = 0;
+  for (uint32_t m = 0; m < 64; ++m)
+    if (oc_valid(m)) {
+      if (ids) ids[n] = m;
+      ++n;
+    }
+  return n;
+}
+
+const char* stencil_oc_name(uint32_t oc) { return oc_name_static(oc); }
+
+int stencil_sample_params(uint32_t oc, int ndim, stencil_dtype_t dtype, uint64_t seed, int k,
+                          stencil_params_t* out) {
+  clear_error();
+  if (!out) SM_FAIL(STENCIL_E_INVAL, "null output");
+  if (!oc_valid(oc)) SM_FAIL(STENCIL_E_OC_INVALID, "OC %u violates Table I", oc);
+  if (ndim != 2 && ndim != 3) SM_FAIL(STENCIL_E_INVAL, "ndim must be 2 or 3");
+  if (dtype != STENCIL_F32 && dtype != STENCIL_F64) SM_FAIL(STENCIL_E_INVAL, "bad dtype");
+  sample_params(oc, ndim, dtype, seed, k, out);
+  return STENCIL_OK;
+}
+
+int stencil_plan_create(stencil_plan_t* plan, int ndim, const int64_t* dims, int order, const uint8_t* access,
+                        const double* coeffs, stencil_dtype_t dtype, uint32_t oc, const stencil_params_t* params) {
+  clear_error();
+  if (!plan) SM_FAIL(STENCIL_E_INVAL, "null plan pointer");
+  *plan = nullptr;
+  if (ndim != 2 && ndim != 3) SM_FAIL(STENCIL_E_INVAL, "ndim must be 2 or 3 (got %d)", ndim);
+  if (order < 1 || order > 4) SM_FAIL(STENCIL_E_INVAL, "order must be in 1..4 (got %d)", order);
+  if (!dims || !access || !coeffs) SM_FAIL(STENCIL_E_INVAL, "null dims/access/coeffs");
+  if (dtype != STENCIL_F32 && dtype != STENCIL_F64) SM_FAIL(STENCIL_E_INVAL, "unknown dtype %d", (int)dtype);
+  for (int k = 0; k < ndim; ++k) {
+    if (dims[k] < 2 * order + 1)
+      SM_FAIL(STENCIL_E_INVAL, "dims[%d]=%lld < 2*order+1=%d", k, (long long)dims[k], 2 * order + 1);
+    if (dims[k] > (1LL << 30)) SM_FAIL(STENCIL_E_INVAL, "dims[%d] too large", k);
+  }
+  {
+    long long vol = 1;
+    for (int k = 0; k < ndim; ++k) vol *= dims[k];
+    if (vol > (1LL << 36)) SM_FAIL(STENCIL_E_INVAL, "grid too large");
+  }
+  const int w = 2 * order + 1;
+  const int tsize = ndim == 3 ? w * w * w : w * w;
+  const int centre = tsize / 2;
+  if (access[centre] != 1) SM_FAIL(STENCIL_E_INVAL, "the centre of the access tensor must be 1 (P:L135)");
+  for (int t = 0; t < tsize; ++t) {
+    if (access[t] > 1) SM_FAIL(STENCIL_E_INVAL, "access tensor must be binary (entry %d = %d)", t, access[t]);
+    if (!access[t] && coeffs[t] != 0.0)
+      SM_FAIL(STENCIL_E_INVAL, "coefficient %d is nonzero where access == 0", t);
+    if (!std::isfinite(coeffs[t])) SM_FAIL(STENCIL_E_INVAL, "coefficient %d is not finite", t);
+  }
+  if (!oc_valid(oc)) SM_FAIL(STENCIL_E_OC_INVALID, "OC %u violates Table I (BM xor CM; RT, PR need ST)", oc);
+  if (params) SM_TRY(validate_params(params));
+
+  std::unique_ptr<stencil_plan_s> P(new stencil_plan_s());
+  P->ndim = ndim;
+  for (int k = 0; k < ndim; ++k) P->dims[k] = dims[k];
+  P->order = order;
+  P->dtype = dtype;
+  P->oc = oc;
+  P->access.assign(access, access + tsize);
+  P->coeffs.assign(coeffs, coeffs + tsize);
+  default_params(oc, ndim, dtype, &P->params);
+  merge_params(params, &P->params);
+  SM_TRY(build_pattern(P.get()));
+  build_view(P.get(), family_of(oc, P->params.smem));
+  SM_TRY(resolve_variant(P.get()));
+  P->src = generate_source(P->pat, P->dtype, P->var);
+  // kernel specialisation (host-only; module load is deferred to first use)
+  SM_TRY(compile_variant(P->pat, P->dtype, P->var, &P->lowered, &P->cubin));
+  *plan = P.release();
+  return STENCIL_OK;
+}
+
+void stencil_plan_destroy(stencil_plan_t plan) { delete plan; }
+
+int stencil_plan_set_stream(stencil_plan_t plan, void* s) {
+  if (!plan) SM_FAIL(STENCIL_E_INVAL, "null plan");
+  plan->stream = (cudaStream_t)s;
+  return STENCIL_OK;
+}
+
+size_t stencil_plan_workspace_bytes(stencil_plan_t plan) {
+  if (!plan) return 0;
+  const int elem = plan->dtype == STENCIL_F64 ? 8 : 4;
+  return (size_t)plan->vdims[0] * plan->vdims[1] * plan->vdims[2] * elem;
+}
+
+int stencil_plan_set_workspace(stencil_plan_t plan, void* p, size_t bytes) {
+  if (!plan) SM_FAIL(STENCIL_E_INVAL, "null plan");
+  if (p && bytes < stencil_plan_workspace_bytes(plan))
+    SM_FAIL(STENCIL_E_INVAL, "workspace of %zu bytes < %zu", bytes, stencil_plan_workspace_bytes(plan));
+  if ((uintptr_t)p % 16) SM_FAIL(STENCIL_E_INVAL, "workspace must be 16-byte aligned");
+  plan->ws = p;
+  plan->ws_bytes = bytes;
+  return STENCIL_OK;
+}
+
+int stencil_plan_info(stencil_plan_t P, stencil_plan_info_t* info) {
+  if (!P || !info) SM_FAIL(STENCIL_E_INVAL, "null argument");
+  memset(info, 0, sizeof *info);
+  info->ndim = P->ndim;
+  info->order = P->order;
+  info->nnz = P->pat.nnz;
+  info->dtype = P->dtype;
+  // extents in the user's axes
+  const Pattern& p = P->pat;
+  if (P->ndim == 2 && (P->var.family == FAM_STREAM || P->var.family == FAM_STREAM_TB)) {
+    int e[6] = {0, 0, p.zlo, p.zhi, p.xlo, p.xhi};
+    memcpy(info->ext, e, sizeof e);
+  } else {
+    int e[6] = {p.zlo, p.zhi, p.ylo, p.yhi, p.xlo, p.xhi};
+    memcpy(info->ext, e, sizeof e);
+  }
+  info->oc = P->oc;
+  info->params = P->params;
+  info->kernel_family = P->var.family;
+  const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+  info->smem_bytes = P->var.smem_bytes(P->pat, elem);
+  info->threads = P->var.threads();
+  info->regs = P->kern.regs;
+  info->uses_tma = P->var.tma ? 1 : 0;
+  long long pts = 1;
+  for (int k = 0; k < 3; ++k) pts *= (P->vdims[k] - 2 * P->frame[k]);
+  info->points = pts;
+  snprintf(info->kernel_name, sizeof info->kernel_name, "%s", P->lowered.c_str());
+  return STENCIL_OK;
+}
+
+int stencil_run(stencil_plan_t plan, const void* in, void* out, int steps) {
+  clear_error();
+  if (!plan) SM_FAIL(STENCIL_E_INVAL, "null plan");
+  return run_device(plan, in, out, steps);
+}
+
+int stencil_run_host(stencil_plan_t P, const void* in_host, void* out_host, int steps) {
+  clear_error();
+  if (!P || !in_host || !out_host) SM_FAIL(STENCIL_E_INVAL, "null argument");
+  const size_t bytes = stencil_plan_workspace_bytes(P);
+  if (!P->h_in_dev) SM_CUDA(cudaMalloc(&P->h_in_dev, bytes));
+  if (!P->h_out_dev) SM_CUDA(cudaMalloc(&P->h_out_dev, bytes));
+  void* saved_ws = P->ws;
+  size_t saved_b = P->ws_bytes;
+  if (!P->ws) {
+    if (!P->h_ws_dev) SM_CUDA(cudaMalloc(&P->h_ws_dev, bytes));
+    P->ws = P->h_ws_dev;
+    P->ws_bytes = bytes;
+  }
+  SM_CUDA(cudaMemcpyAsync(P->h_in_dev, in_host, bytes, cudaMemcpyHostToDevice, P->stream));
+  int rc = run_device(P, P->h_in_dev, P->h_out_dev, steps);
+  P->ws = saved_ws;
+  P->ws_bytes = saved_b;
+  if (rc != STENCIL_OK) return rc;
+  SM_CUDA(cudaMemcpyAsync(out_host, P->h_out_dev, bytes, cudaMemcpyDeviceToHost, P->stream));
+  SM_CUDA(cudaStreamSynchronize(P->stream));
+  return STENCIL_OK;
+}
+
+int stencil_fill_field(void* dev, stencil_dtype_t dtype, int ndim, const int64_t* box_dims, const int64_t* origin,
+                       const int64_t* global_dims, uint64_t seed, int kind, void* stream) {
+  clear_error();
+  if (!dev || !box_dims || !global_dims) SM_FAIL(STENCIL_E_INVAL, "null argument");
+  if (ndim < 1 || ndim > 3) SM_FAIL(STENCIL_E_INVAL, "ndim must be 1..3");
+  if (dtype != STENCIL_F32 && dtype != STENCIL_F64) SM_FAIL(STENCIL_E_INVAL, "bad dtype");
+  if (kind != 0 && kind != 1) SM_FAIL(STENCIL_E_INVAL, "kind must be 0 or 1");
+  int64_t b[3] = {1, 1, 1}, o[3] = {0, 0, 0}, g[3] = {1, 1, 1};
+  for (int k = 0; k < ndim; ++k) {
+    b[3 - ndim + k] = box_dims[k];
+    o[3 - ndim + k] = origin ? origin[k] : 0;
+    g[3 - ndim + k] = global_dims[k];
+    if (b[3 - ndim + k] < 0 || o[3 - ndim + k] < 0 || o[3 - ndim + k] + b[3 - ndim + k] > g[3 - ndim + k])
+      SM_FAIL(STENCIL_E_INVAL, "box outside the global grid on axis %d", k);
+  }
+  return launch_fill(dev, dtype, b, o, g, seed, kind, (cudaStream_t)stream);
+}
+
+int stencil_slab_range(int64_t nz_global, int rank, int nranks, int64_t* z_begin, int64_t* z_end) {
+  clear_error();
+  if (nranks < 1 || rank < 0 || rank >= nranks || !z_begin || !z_end || nz_global < nranks)
+    SM_FAIL(STENCIL_E_INVAL, "bad slab arguments");
+  const int64_t base = nz_global / nranks, rem = nz_global % nranks;
+  *z_begin = rank * base + std::min<int64_t>(rank, rem);
+  *z_end = *z_begin + base + (rank < rem ? 1 : 0);
+  return STENCIL_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,361 @@
+// codegen.cpp -- kernel specialisation.
+//
+// The paper generates one "stencil program" per stencil and OC (P:L25,
+// P:L234). Here the generated part is only DATA: a descriptor struct holding
+// the offsets (as a dense index table over the stencil's bounding box) and the
+// coefficients rounded to the plan dtype, written as exact hex-float literals.
+// The hand-written kernel templates of kernels/stencil_kernels.cuh are compiled
+// against it with NVRTC for sm_100a. Cubins are cached per process and on disk.
+#include <nvrtc.h>
+#include <sys/stat.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <fstream>
+#include <mutex>
+#include <sstream>
+
+#include "internal.h"
+
+namespace smart_rt {
+
+#include "kernels_src.inc"   // static const char kKernelsSrc[] (generated at build time)
+
+namespace {
+
+std::mutex g_mu;
+std::map<std::string, CUmodule> g_modules;          // source -> loaded module
+std::map<std::string, std::pair<std::string, std::vector<char>>> g_cubins;  // source -> (lowered, cubin)
+
+uint64_t fnv1a(const std::string& s) {
+  uint64_t h = 1469598103934665603ull;
+  for (unsigned char c : s) { h ^= c; h *= 1099511628211ull; }
+  return h;
+}
+
+std::string cache_dir() {
+  const char* d = getenv("STENCIL_CACHE_DIR");
+  std::string dir;
+  if (d && *d) dir = d;
+  else {
+    const char* home = getenv("HOME");
+    dir = std::string(home && *home ? home : "/tmp") + "/.cache/stencilmart";
+  }
+  return dir;
+}
+
+void mkdirs(const std::string& path) {
+  std::string cur;
+  std::stringstream ss(path);
+  std::string part;
+  if (!path.empty() && path[0] == '/') cur = "/";
+  while (std::getline(ss, part, '/')) {
+    if (part.empty()) continue;
+    cur += part + "/";
+    mkdir(cur.c_str(), 0755);
+  }
+}
+
+bool read_file(const std::string& p, std::vector<char>* out) {
+  std::ifstream f(p, std::ios::binary);
+  if (!f) return false;
+  out->assign(std::istreambuf_iterator<char>(f), std::istreambuf_iterator<char>());
+  return !out->empty();
+}
+
+void write_file_atomic(const std::string& p, const char* data, size_t n) {
+  std::string tmp = p + ".tmp" + std::to_string(getpid());
+  std::ofstream f(tmp, std::ios::binary);
+  if (!f) return;
+  f.write(data, (std::streamsize)n);
+  f.close();
+  rename(tmp.c_str(), p.c_str());
+}
+
+std::string hexfloat(double v, bool f32) {
+  char buf[64];
+  if (f32) {
+    float x = (float)v;                       // round-to-nearest-even, once (C-19)
+    if (x == 0.0f) return std::signbit(x) ? "-0.0f" : "0.0f";
+    snprintf(buf, sizeof buf, "%af", (double)x);
+  } else {
+    if (v == 0.0) return std::signbit(v) ? "-0.0" : "0.0";
+    snprintf(buf, sizeof buf, "%a", v);
+  }
+  return buf;
+}
+
+}  // namespace
+
+std::string Variant::name_expr(const char* desc) const {
+  char b[256];
+  const char* tf = tma ? "true" : "false";
+  const char* cmf = cm ? "true" : "false";
+  switch (family) {
+    case FAM_NAIVE:
+      snprintf(b, sizeof b, "smart::k_naive<%s, %d, %d, %d, %s>", desc, bx, by, m, cmf);
+      break;
+    case FAM_TILED:
+      snprintf(b, sizeof b, "smart::k_tiled<%s, %d, %d, %d, %d, %d, %s, %d, %s>", desc, bx, by, bz, vx, m,
+               cmf, tt, tf);
+      break;
+    case FAM_STREAM:
+      snprintf(b, sizeof b, "smart::k_stream<%s, %d, %d, %d, %d, %s, %s, %d, %s>", desc, bx, by, vx, m, cmf,
+               rt ? "true" : "false", ns, tf);
+      break;
+    default:
+      snprintf(b, sizeof b, "smart::k_stream_tb<%s, %d, %d, %d, %d, %s, %s, %d, %d, %s>", desc, bx, by, vx,
+               m, cmf, rt ? "true" : "false", ns, tt, tf);
+      break;
+  }
+  return b;
+}
+
+int Variant::threads() const {
+  switch (family) {
+    case FAM_NAIVE: return bx * by;
+    default: return (bx / vx) * by;
+  }
+}
+
+static int roundup(int a, int b) { return (a + b - 1) / b * b; }
+
+// Mirrors TiledCfg / StreamCfg of stencil_kernels.cuh.
+int Variant::smem_bytes(const Pattern& p, int elem) const {
+  const int aln = std::max(16 / elem, vx);
+  if (family == FAM_TILED) {
+    const int xoff = roundup(tt * p.xlo, vx);
+    const int lx = roundup(xoff + bx + tt * p.xhi, aln);
+    const int ly = by * m + tt * (p.ylo + p.yhi);
+    const int lz = bz + tt * (p.zlo + p.zhi);
+    const int buf = roundup(lx * ly * lz * elem, 128) / elem;
+    return (tt > 1 ? 2 : 1) * buf * elem + 128;
+  }
+  if (family == FAM_STREAM) {
+    const int xoff = roundup(p.xlo, vx);
+    const int lx = roundup(xoff + bx + p.xhi, aln);
+    const int ly = by * m + p.ylo + p.yhi;
+    const int plane = roundup(lx * ly * elem, 128) / elem;
+    const int nz = p.zlo + p.zhi + 1;
+    const int nring = (rt ? 1 : nz) + ns - 1;
+    return nring * plane * elem + 8 * nring + 128;
+  }
+  return 0;
+}
+
+// Op table of a variant (format documented at run_gather in stencil_kernels.cuh).
+// Loops are ordered so that every accumulator receives its FMAs in
+// lexicographic (dz, dy, dx) order -- the canonical chain of every OC.
+static std::vector<uint32_t> encode_ops(const Pattern& pat, const Variant& v) {
+  const int NZ = pat.zlo + pat.zhi + 1, NY = pat.ylo + pat.yhi + 1, NX = pat.xlo + pat.xhi + 1;
+  std::vector<int> idx((size_t)NZ * NY * NX, -1);
+  for (int i = 0; i < pat.nnz; ++i)
+    idx[((size_t)(pat.dz[i] + pat.zlo) * NY + pat.dy[i] + pat.ylo) * NX + pat.dx[i] + pat.xlo] = i;
+  auto cidx = [&](int zi, int yi, int xi) {
+    if (zi < 0 || zi >= NZ || yi < 0 || yi >= NY || xi < 0 || xi >= NX) return -1;
+    return idx[((size_t)zi * NY + yi) * NX + xi];
+  };
+  const int VX = v.family == FAM_NAIVE ? 1 : v.vx;
+  const int M = v.m, BY = v.by;
+  const bool scatter = v.rt && (v.family == FAM_STREAM || v.family == FAM_STREAM_TB);
+  const int KLO = -((pat.xlo + VX - 1) / VX), KHI = (VX - 1 + pat.xhi) / VX;
+  auto load = [](int zi, int j, int kv) {
+    return (uint32_t)(zi & 15) | ((uint32_t)(j + 128) & 255) << 4 | ((uint32_t)(kv + 8) & 15) << 12;
+  };
+  auto fma = [](int id, int e, int vv, int m, int zi) {
+    return 0x80000000u | (uint32_t)id | (uint32_t)e << 10 | (uint32_t)vv << 12 | (uint32_t)m << 14 |
+           (uint32_t)zi << 17;
+  };
+  std::vector<uint32_t> ops, f;
+  auto window = [&](int zsel, int j_rel, int kv, int zi_lo, int zi_hi, int m_lo, int m_hi, int jbase) {
+    // FMAs fed by window (row j_rel, vector kv); jbase = j_rel - (row of output m_lo's dy = 0)
+    f.clear();
+    for (int zi = zi_lo; zi < zi_hi; ++zi)
+      for (int m = m_lo; m < m_hi; ++m)
+        for (int vv = 0; vv < VX; ++vv)
+          for (int e = 0; e < VX; ++e) {
+            const int dyi = (v.cm ? jbase : jbase - m) + pat.ylo;
+            const int id = cidx(zi, dyi, kv * VX + e - vv + pat.xlo);
+            if (id >= 0) f.push_back(fma(id, e, vv, m, zi));
+          }
+    if (!f.empty()) {
+      ops.push_back(load(zsel, j_rel, kv));
+      ops.insert(ops.end(), f.begin(), f.end());
+    }
+  };
+  if (!v.cm) {
+    if (!scatter) {
+      for (int zi = 0; zi < NZ; ++zi)
+        for (int j = -pat.ylo; j < M + pat.yhi; ++j)
+          for (int kv = KLO; kv <= KHI; ++kv) window(zi, j, kv, zi, zi + 1, 0, M, j);
+    } else {
+      for (int j = -pat.ylo; j < M + pat.yhi; ++j)
+        for (int kv = KLO; kv <= KHI; ++kv) window(0, j, kv, 0, NZ, 0, M, j);
+    }
+  } else {
+    if (!scatter) {
+      for (int zi = 0; zi < NZ; ++zi)
+        for (int m = 0; m < M; ++m)
+          for (int j = -pat.ylo; j <= pat.yhi; ++j)
+            for (int kv = KLO; kv <= KHI; ++kv) window(zi, m * BY + j, kv, zi, zi + 1, m, m + 1, j);
+    } else {
+      for (int m = 0; m < M; ++m)
+        for (int j = -pat.ylo; j <= pat.yhi; ++j)
+          for (int kv = KLO; kv <= KHI; ++kv) window(0, m * BY + j, kv, 0, NZ, m, m + 1, j);
+    }
+  }
+  return ops;
+}
+
+std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
+  const bool f32 = dtype == STENCIL_F32;
+  const int NZ = pat.zlo + pat.zhi + 1, NY = pat.ylo + pat.yhi + 1, NX = pat.xlo + pat.xhi + 1;
+  std::vector<int> idx((size_t)NZ * NY * NX, -1);
+  for (int i = 0; i < pat.nnz; ++i) {
+    const int zi = pat.dz[i] + pat.zlo, yi = pat.dy[i] + pat.ylo, xi = pat.dx[i] + pat.xlo;
+    idx[((size_t)zi * NY + yi) * NX + xi] = i;
+  }
+  std::ostringstream o;
+  o << "// generated stencil descriptor: nnz=" << pat.nnz << "\n";
+  o << "#include \"stencil_kernels.cuh\"\n";
+  o << "namespace gen {\n";
+  o << "__device__ constexpr short g_idx[" << NZ << "][" << NY << "][" << NX << "] = {";
+  for (int z = 0; z < NZ; ++z) {
+    o << "{";
+    for (int y = 0; y < NY; ++y) {
+      o << "{";
+      for (int x = 0; x < NX; ++x) o << idx[((size_t)z * NY + y) * NX + x] << (x + 1 < NX ? "," : "");
+      o << "}" << (y + 1 < NY ? "," : "");
+    }
+    o << "}" << (z + 1 < NZ ? "," : "");
+  }
+  o << "};\n";
+  const char* T = f32 ? "float" : "double";
+  o << "__device__ constexpr " << T << " g_coef[" << pat.nnz << "] = {";
+  for (int i = 0; i < pat.nnz; ++i) o << hexfloat(pat.c[i], f32) << (i + 1 < pat.nnz ? "," : "");
+  o << "};\n";
+  const std::vector<uint32_t> ops = encode_ops(pat, v);
+  o << "__device__ constexpr unsigned g_ops[" << std::max<size_t>(ops.size(), 1) << "] = {";
+  for (size_t i = 0; i < ops.size(); ++i) o << ops[i] << "u" << (i + 1 < ops.size() ? "," : "");
+  if (ops.empty()) o << "0u";
+  o << "};\n";
+  o << "struct S {\n  typedef " << T << " T;\n";
+  o << "  static constexpr int NNZ = " << pat.nnz << ", ZLO = " << pat.zlo << ", ZHI = " << pat.zhi
+    << ", YLO = " << pat.ylo << ", YHI = " << pat.yhi << ", XLO = " << pat.xlo << ", XHI = " << pat.xhi
+    << ", NZ = " << NZ << ", NY = " << NY << ", NX = " << NX << ";\n";
+  o << "  static __device__ __forceinline__ constexpr int idx(int z, int y, int x) { return g_idx[z][y][x]; }\n";
+  o << "  static __device__ __forceinline__ constexpr T coef(int i) { return g_coef[i]; }\n";
+  o << "  static constexpr int NOPS = " << ops.size() << ";\n";
+  o << "  static __device__ __forceinline__ constexpr unsigned op(int i) { return g_ops[i]; }\n";
+  o << "};\n}  // namespace gen\n";
+  o << "// variant: " << v.name_expr("gen::S") << "\n";
+  return o.str();
+}
+
+int compile_variant(const Pattern& pat, int dtype, const Variant& v, std::string* lowered,
+                    std::vector<char>* cubin) {
+  const std::string src = generate_source(pat, dtype, v);
+  const std::string expr = "&" + v.name_expr("gen::S");
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    auto it = g_cubins.find(src);
+    if (it != g_cubins.end()) {
+      *lowered = it->second.first;
+      *cubin = it->second.second;
+      return STENCIL_OK;
+    }
+  }
+  const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "-default-device",
+                        "--extra-device-vectorization"};
+  const int nopt = sizeof(opts) / sizeof(opts[0]);
+  int nv_major = 0, nv_minor = 0;
+  nvrtcVersion(&nv_major, &nv_minor);
+  std::string key_str = src + "|" + kKernelsSrc + "|";
+  for (int i = 0; i < nopt; ++i) key_str += std::string(opts[i]) + " ";
+  key_str += std::to_string(nv_major) + "." + std::to_string(nv_minor);
+  char hname[32];
+  snprintf(hname, sizeof hname, "%016llx", (unsigned long long)fnv1a(key_str));
+  const std::string dir = cache_dir();
+  const std::string base = dir + "/" + hname;
+
+  // disk cache
+  std::vector<char> bin, nm;
+  if (read_file(base + ".cubin", &bin) && read_file(base + ".name", &nm)) {
+    *lowered = std::string(nm.begin(), nm.end());
+    *cubin = bin;
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_cubins[src] = {*lowered, *cubin};
+    return STENCIL_OK;
+  }
+
+  nvrtcProgram prog;
+  const char* hdr_src[] = {kKernelsSrc};
+  const char* hdr_name[] = {"stencil_kernels.cuh"};
+  nvrtcResult r = nvrtcCreateProgram(&prog, src.c_str(), "stencil_gen.cu", 1, hdr_src, hdr_name);
+  if (r != NVRTC_SUCCESS) SM_FAIL(STENCIL_E_NVRTC, "nvrtcCreateProgram: %s", nvrtcGetErrorString(r));
+  nvrtcAddNameExpression(prog, expr.c_str());
+  r = nvrtcCompileProgram(prog, nopt, opts);
+  if (r != NVRTC_SUCCESS) {
+    size_t ls = 0;
+    nvrtcGetProgramLogSize(prog, &ls);
+    std::string log(ls, '\0');
+    nvrtcGetProgramLog(prog, &log[0]);
+    nvrtcDestroyProgram(&prog);
+    if (log.size() > 3000) log = log.substr(0, 3000) + "...";
+    SM_FAIL(STENCIL_E_NVRTC, "NVRTC compile of %s failed: %s", expr.c_str(), log.c_str());
+  }
+  const char* low = nullptr;
+  nvrtcGetLoweredName(prog, expr.c_str(), &low);
+  *lowered = low ? low : "";
+  size_t cs = 0;
+  nvrtcGetCUBINSize(prog, &cs);
+  cubin->resize(cs);
+  nvrtcGetCUBIN(prog, cubin->data());
+  nvrtcDestroyProgram(&prog);
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_cubins[src] = {*lowered, *cubin};
+  }
+  mkdirs(dir);
+  write_file_atomic(base + ".cubin", cubin->data(), cubin->size());
+  write_file_atomic(base + ".name", lowered->data(), lowered->size());
+  return STENCIL_OK;
+}
+
+int load_kernel(const std::string& key_src, const std::vector<char>& cubin, const std::string& lowered,
+                int smem, Kernel* out) {
+  const Driver* d = nullptr;
+  SM_TRY(get_driver(&d));
+  SM_CUDA(cudaFree(nullptr));   // make the primary context current
+  CUmodule mod = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    auto it = g_modules.find(key_src);
+    if (it != g_modules.end()) mod = it->second;
+  }
+  if (!mod) {
+    CUresult r = d->moduleLoadData(&mod, cubin.data());
+    if (r != CUDA_SUCCESS) SM_FAIL(STENCIL_E_CUDA, "cuModuleLoadData: %s", cu_errstr(r));
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_modules[key_src] = mod;
+  }
+  CUfunction fn = nullptr;
+  CUresult r = d->moduleGetFunction(&fn, mod, lowered.c_str());
+  if (r != CUDA_SUCCESS) SM_FAIL(STENCIL_E_CUDA, "cuModuleGetFunction(%s): %s", lowered.c_str(), cu_errstr(r));
+  if (smem > 48 * 1024) {
+    r = d->funcSetAttribute(fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, smem);
+    if (r != CUDA_SUCCESS)
+      SM_FAIL(STENCIL_E_OC_INFEASIBLE, "shared memory %d B not available: %s", smem, cu_errstr(r));
+  }
+  out->fn = fn;
+  d->funcGetAttribute(&out->regs, CU_FUNC_ATTRIBUTE_NUM_REGS, fn);
+  d->funcGetAttribute(&out->local_bytes, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, fn);
+  return STENCIL_OK;
+}
+
+}  // namespace smart_rt

