@@ -313,7 +313,9 @@ template <class S, int BX, int BY, int BZ, int VX, int M, bool CM, int TT>
 struct TiledCfg {
   typedef typename S::T T;
   static constexpr int ALN = (16 / (int)sizeof(T)) > VX ? (16 / (int)sizeof(T)) : VX;
-  static constexpr int XOFF = ((TT * S::XLO + VX - 1) / VX) * VX;       // smem col of tile x origin
+  // smem column of the tile's x origin; a multiple of ALN so the TMA box starts
+  // on a 16-byte boundary (cp.async.bulk.tensor faults on a misaligned x start)
+  static constexpr int XOFF = ((TT * S::XLO + ALN - 1) / ALN) * ALN;
   static constexpr int LX = ((XOFF + BX + TT * S::XHI + ALN - 1) / ALN) * ALN;
   static constexpr int LY = BY * M + TT * (S::YLO + S::YHI);
   static constexpr int LZ = BZ + TT * (S::ZLO + S::ZHI);
@@ -444,7 +446,7 @@ template <class S, int BX, int BY, int VX, int M, bool CM, bool RT, int NS>
 struct StreamCfg {
   typedef typename S::T T;
   static constexpr int ALN = (16 / (int)sizeof(T)) > VX ? (16 / (int)sizeof(T)) : VX;
-  static constexpr int XOFF = ((S::XLO + VX - 1) / VX) * VX;
+  static constexpr int XOFF = ((S::XLO + ALN - 1) / ALN) * ALN;   // 16-byte aligned box start
   static constexpr int LX = ((XOFF + BX + S::XHI + ALN - 1) / ALN) * ALN;
   static constexpr int LY = BY * M + S::YLO + S::YHI;
   static constexpr int PLANE = ((LX * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);

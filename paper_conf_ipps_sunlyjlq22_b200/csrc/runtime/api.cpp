@@ -226,11 +226,11 @@ static TmaBox tma_box(const Variant& v, const Pattern& p, int elem) {
   const int aln = std::max(16 / elem, v.vx);
   auto ru = [](int a, int b) { return (a + b - 1) / b * b; };
   if (v.family == FAM_TILED) {
-    const int xoff = ru(v.tt * p.xlo, v.vx);
+    const int xoff = ru(v.tt * p.xlo, aln);
     return {ru(xoff + v.bx + v.tt * p.xhi, aln), v.by * v.m + v.tt * (p.ylo + p.yhi),
             v.bz + v.tt * (p.zlo + p.zhi)};
   }
-  const int xoff = ru(p.xlo, v.vx);
+  const int xoff = ru(p.xlo, aln);
   return {ru(xoff + v.bx + p.xhi, aln), v.by * v.m + p.ylo + p.yhi, 1};
 }
 

@@ -129,7 +129,7 @@ static int roundup(int a, int b) { return (a + b - 1) / b * b; }
 int Variant::smem_bytes(const Pattern& p, int elem) const {
   const int aln = std::max(16 / elem, vx);
   if (family == FAM_TILED) {
-    const int xoff = roundup(tt * p.xlo, vx);
+    const int xoff = roundup(tt * p.xlo, aln);
     const int lx = roundup(xoff + bx + tt * p.xhi, aln);
     const int ly = by * m + tt * (p.ylo + p.yhi);
     const int lz = bz + tt * (p.zlo + p.zhi);
@@ -137,7 +137,7 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     return (tt > 1 ? 2 : 1) * buf * elem + 128;
   }
   if (family == FAM_STREAM) {
-    const int xoff = roundup(p.xlo, vx);
+    const int xoff = roundup(p.xlo, aln);
     const int lx = roundup(xoff + bx + p.xhi, aln);
     const int ly = by * m + p.ylo + p.yhi;
     const int plane = roundup(lx * ly * elem, 128) / elem;
