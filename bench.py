@@ -1,0 +1,403 @@
+#!/usr/bin/env python
+"""bench.py -- GStencil/s and % of HBM roofline per OC on B200 (BASELINE.json metric).
+
+Default workload (BASELINE.json configs[1], "C2"): the 3-D 7-point heat stencil
+(order 1) on a 512^3 fp64 grid, 10 time steps, under every OC of Table I.
+
+What one run does (one process per GPU; torchrun for N > 1):
+  1. label pass: stencil_oc_sweep over the 30 OCs with the
+     library's seeded settings; its per-OC times give "per_oc" (GStencil/s and
+     HBM fraction of every OC) and the label (best OC + its setting);
+  2. W warm-up steps, then K timed steps of the production path: one timed
+     step = stencil_run of the config's 10 time steps with the labelled OC,
+     inputs resident in HBM (1 GiB per grid >> 126 MB L2, so no flush is
+     needed), bracketed by barrier + synchronize, CUDA events on the plan's
+     stream, max over ranks;
+  3. roofline of the dominant kernel (the labelled OC's sweep kernel): bytes a
+     launch must move (read + write the grid once: 16 B / point in fp64, for
+     every fused step count) / its average launch duration, from CUDA events
+     around each launch over the timed region;
+  4. e2e: the same metric through stencil_run_host (pinned host buffers in,
+     H2D + 10 steps + D2H inside the timed region);
+  5. cpu_baseline: the oracle (oracle/, plain C loops, OpenMP) on a bounded
+     sample of the same workload on this host's cores (rank 0, N = 1 only).
+`--impl reference` times only the oracle (the "reference arm" of this tier).
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "GStencil/s and % of HBM roofline per OC at 1/2/4/8 B200"
+HBM_SPEC_GBS = 8000.0
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d.get("hbm_gbs", 6650.0)), "measured"
+    return 6650.0, "fallback"
+
+
+WORKLOADS = {
+    "C2": "C2: 3-D 7-point heat star (order 1), 512^3 fp64 per GPU, 10 time steps, all 30 OCs swept, best OC timed",
+    "C3": "C3: 3-D 25-point star (order 4), 768^3 fp32 per GPU, 10 time steps, ST/RT family swept, best OC timed",
+    "C4": "C4: 3-D 125-point box (order 2), 512^3 fp64 per GPU, 10 time steps, TB vs tiling family swept",
+    "C1": "C1: 2-D 5-point heat star (order 1), 256^2 fp64, 10 time steps, naive OC",
+}
+
+
+def _env_rank():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+class ClockSampler:
+    """NVML SM clock + throttle reasons sampled during the timed region."""
+
+    def __init__(self, index: int):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        self._t = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        nv = self.nv
+        names = {
+            "hw_slowdown": getattr(nv, "nvmlClocksEventReasonHwSlowdown", 0x8),
+            "hw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonHwThermalSlowdown", 0x40),
+            "sw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonSwThermalSlowdown", 0x20),
+            "sw_power_cap": getattr(nv, "nvmlClocksEventReasonSwPowerCap", 0x4),
+            "hw_power_brake_slowdown": getattr(nv, "nvmlClocksEventReasonHwPowerBrakeSlowdown", 0x80),
+        }
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for k, bit in names.items():
+                    if r & bit:
+                        self.reasons.add(k)
+            except Exception:
+                pass
+            self._stop.wait(0.02)
+
+    def __enter__(self):
+        if self.nv:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def result(self):
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def _config(name: str):
+    import stencil_inputs as si
+    C = dict(si.CONFIGS[name])
+    acc, c = si.config_stencil(C["stencil"])
+    return C, acc, c
+
+
+def _ocs_for(name: str, sm):
+    if name == "C2":
+        return sm.oc_list()
+    if name == "C3":
+        return [o for o in sm.oc_list() if o & sm.OC_ST and not o & sm.OC_TB]
+    if name == "C4":
+        return [o for o in sm.oc_list() if not o & sm.OC_ST or o & sm.OC_RT]
+    if name == "C1":
+        return [0]
+    return sm.oc_list()
+
+
+def cpu_oracle_sample(name: str, budget_s: float = 12.0):
+    """Time the oracle (as it stands) on a bounded z-slab of the workload."""
+    import oracle
+    import stencil_inputs as si
+    C, acc, c = _config(name)
+    dims, steps, dtype = C["dims"], C["steps"], C["dtype"]
+    r = (acc.shape[0] - 1) // 2
+    threads = oracle.max_threads()
+    if len(dims) == 2:
+        u = si.make_field(dims, C["seed"], dtype)
+        t0 = time.perf_counter()
+        oracle.sweep(u, acc, c, steps, dtype=dtype)
+        dt = time.perf_counter() - t0
+        pts = (dims[0] - 2 * r) * (dims[1] - 2 * r) * steps
+        return {"value": pts / dt / 1e9, "unit": "GStencil/s", "cores": threads, "kind": "oracle",
+                "sample": f"full C1 grid {dims}, {steps} steps, {dt:.2f} s", "seconds": dt}
+    # probe with a thin slab, then size the sample to ~budget_s
+    nz = 2 * r + 8
+    u = si.make_field((nz, dims[1], dims[2]), C["seed"], dtype, global_dims=dims)
+    t0 = time.perf_counter()
+    oracle.sweep(u, acc, c, 1, dtype=dtype)
+    per_plane = (time.perf_counter() - t0) / (nz - 2 * r)
+    full = dims[0] - 2 * r
+    if per_plane * full * steps <= budget_s:          # the whole workload fits the budget
+        planes, s_steps = full, steps
+    else:
+        s_steps = max(1, min(steps, int(budget_s / max(per_plane * full, 1e-9))))
+        planes = int(max(8, min(full, budget_s / max(per_plane, 1e-9) / s_steps)))
+    u = si.make_field((planes + 2 * r, dims[1], dims[2]), C["seed"], dtype, global_dims=dims)
+    t0 = time.perf_counter()
+    oracle.sweep(u, acc, c, s_steps, dtype=dtype)
+    dt = time.perf_counter() - t0
+    pts = planes * (dims[1] - 2 * r) * (dims[2] - 2 * r) * s_steps
+    return {"value": pts / dt / 1e9, "unit": "GStencil/s", "cores": threads, "kind": "oracle",
+            "sample": (f"{planes}+{2 * r} planes x {dims[1]}x{dims[2]} of the {name} grid, {s_steps} step(s), "
+                       f"{dt:.2f} s; rate per interior update"), "seconds": dt}
+
+
+def run_reference(args):
+    rank, world, _ = _env_rank()
+    if rank != 0:
+        return 0
+    name = args.config
+    budget = max(2.0, min(60.0, 150.0 / max(1, args.steps + args.warmup)))
+    vals = []
+    cb = None
+    for i in range(args.warmup + args.steps):
+        cb = cpu_oracle_sample(name, budget)
+        if i >= args.warmup:
+            vals.append(cb["value"])
+    v = statistics.mean(vals)
+    C, acc, c = _config(name)
+    pts = 1
+    r = (acc.shape[0] - 1) // 2
+    for d in C["dims"]:
+        pts *= d - 2 * r
+    ms = pts * C["steps"] / (v * 1e9) * 1e3
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "GStencil/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": C["dtype"], "data": "synthetic",
+        "config": {"workload": WORKLOADS.get(name, name), "grid": list(C["dims"]), "time_steps": C["steps"],
+                   "note": "oracle timed on a bounded z-slab sample; ms_per_step extrapolated to the full grid"},
+        "cpu_baseline": {k: cb[k] for k in ("kind", "cores", "sample")} | {"value": v, "unit": "GStencil/s"},
+        "e2e": {"value": v, "unit": "GStencil/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def _traffic_from_profiles(kernel_name: str):
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    try:
+        d = json.load(open(p))
+        e = d.get(kernel_name)
+        return float(e["dram_bytes_per_launch"]) if e else None
+    except Exception:
+        return None
+
+
+def run_impl(args):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_sunlyjlq22_b200 as sm
+
+    rank, world, local = _env_rank()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    sm.lib()
+    name = args.config
+    C, acc, c = _config(name)
+    dims, steps, dtype = tuple(C["dims"]), C["steps"], C["dtype"]
+    tdt = torch.float64 if dtype == "f64" else torch.float32
+    elem = 8 if dtype == "f64" else 4
+    peak, peak_kind = _peaks()
+
+    x = torch.empty(dims, dtype=tdt, device=dev)
+    # every rank holds its own slab of a global grid of depth sum(nz) (weak scaling)
+    gdims = (dims[0] * world,) + dims[1:] if len(dims) == 3 else dims
+    origin = (dims[0] * rank, 0, 0) if len(dims) == 3 else (0, 0)
+    sm.fill_field(x, C["seed"], 0, origin=origin, global_dims=gdims)
+    y = torch.empty_like(x)
+    stream = torch.cuda.current_stream()
+
+    # ---- 1. label pass: every OC of the family, seeded settings (a8)
+    base_plan = sm.Plan(dims, acc, c, dtype, 0)
+    info0 = base_plan.info
+    pts = info0["points"]
+    ocs = _ocs_for(name, sm)
+    t_sw = time.time()
+    if args.settings > 0 and len(ocs) > 1:
+        sweep = base_plan.oc_sweep(x, y, steps=steps, settings_per_oc=args.settings, reps=3, seed=args.seed)
+    else:
+        sweep = {"oc_ids": sm.oc_list(), "times_ms": [math.inf] * sm.NUM_OC,
+                 "best_params": [{}] * sm.NUM_OC, "best_oc": ocs[0]}
+    sweep_s = time.time() - t_sw
+    per_oc = {}
+    best_oc, best_t, best_p = None, math.inf, None
+    for oc, t, p in zip(sweep["oc_ids"], sweep["times_ms"], sweep["best_params"]):
+        if oc not in ocs:
+            continue
+        gs = sm.gstencil_per_s(pts, steps, t) if math.isfinite(t) else None
+        per_oc[sm.oc_name(oc)] = {
+            "ms": round(t, 4) if math.isfinite(t) else None,
+            "gstencil_s": round(gs, 2) if gs else None,
+            "hbm_frac_of_measured": round(gs * 2 * elem / peak, 4) if gs else None,
+            "hbm_frac_of_spec": round(gs * 2 * elem / HBM_SPEC_GBS, 4) if gs else None,
+            "infeasible": not math.isfinite(t),
+        }
+        if math.isfinite(t) and t < best_t:
+            best_oc, best_t, best_p = oc, t, p
+    if best_oc is None:
+        best_oc, best_p = ocs[0], None
+    if world > 1:   # every rank must run the same OC: take rank 0's label
+        obj = [best_oc, best_p]
+        dist.broadcast_object_list(obj, src=0)
+        best_oc, best_p = obj
+
+    plan = sm.Plan(dims, acc, c, dtype, best_oc, best_p or None)
+    pinfo = plan.info
+
+    # ---- 2. warm-up + timed steps
+    for _ in range(args.warmup):
+        plan.run(x, y, steps)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    launches0 = sm.launch_count()
+    plan.set_timing(True)
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        e0.record(stream)
+        for _ in range(args.steps):
+            plan.run(x, y, steps)
+        e1.record(stream)
+        torch.cuda.synchronize()
+    launches = sm.launch_count() - launches0
+    kern_ms, kern_n = plan.kernel_time()
+    plan.set_timing(False)
+    total_ms = e0.elapsed_time(e1)
+    if world > 1:
+        t = torch.tensor([total_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+        dist.barrier()
+    ms_per_step = total_ms / args.steps
+    value = pts * steps * world / (ms_per_step * 1e-3) / 1e9
+
+    # ---- 3. roofline of the dominant kernel (the labelled OC's sweep kernel)
+    T = pinfo["params"]["tb_steps"] if best_oc & sm.OC_TB else 1
+    bytes_per_launch = pts * 2 * elem          # read + write each interior point once per launch
+    avg_launch_ms = kern_ms / max(kern_n, 1)
+    achieved = bytes_per_launch / (avg_launch_ms * 1e-3) / 1e9
+    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "traffic": _traffic_from_profiles(pinfo["kernel_name"]),
+                "peak_kind": peak_kind, "kernel": pinfo["kernel_name"][:100], "launch_ms": round(avg_launch_ms, 4),
+                "kernel_share_of_step": round(kern_ms / max(total_ms, 1e-9), 4),
+                "bytes_per_launch": bytes_per_launch, "time_steps_per_launch": T,
+                "frac_of_spec_8tbs": round(achieved / HBM_SPEC_GBS, 4)}
+
+    # ---- 4. e2e through the public API with host buffers
+    e2e = None
+    if not args.no_e2e:
+        hin = torch.empty(dims, dtype=tdt, pin_memory=True)
+        hin.copy_(x.cpu())
+        hout = torch.empty_like(hin).pin_memory()
+        plan.run_host(hin, hout, steps)   # warm (allocates the plan's device buffers)
+        n_e2e = max(1, min(3, args.steps))
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(n_e2e):
+            plan.run_host(hin, hout, steps)
+        torch.cuda.synchronize()
+        e2e_ms = (time.perf_counter() - t0) * 1e3 / n_e2e
+        if world > 1:
+            t = torch.tensor([e2e_ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e2e_ms = float(t.item())
+        nbytes = x.numel() * elem
+        e2e = {"value": round(pts * steps * world / (e2e_ms * 1e-3) / 1e9, 3), "unit": "GStencil/s",
+               "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes, "ms_per_step": round(e2e_ms, 3)}
+        del hin, hout
+
+    # ---- 5. CPU oracle beside it (rank 0, N = 1)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cb = cpu_oracle_sample(name, args.cpu_budget)
+        cpu = {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample")}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 2), "unit": "GStencil/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": dtype,
+            "data": "synthetic",
+            "config": {"workload": WORKLOADS.get(name, name), "grid_per_gpu": list(dims),
+                       "global_grid": list(gdims), "time_steps_per_step": steps,
+                       "stencil": C["stencil"], "oc": sm.oc_name(best_oc), "params": pinfo["params"],
+                       "parallelism": f"replicas x{world}" if world > 1 else "single GPU",
+                       "l2": "inputs (grid bytes) larger than the 126 MB L2; no flush needed"},
+            "roofline": roofline,
+            "hbm_frac_of_measured": round(value / world * 2 * elem / peak, 4),
+            "hbm_frac_of_spec": round(value / world * 2 * elem / HBM_SPEC_GBS, 4),
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "clocks": clk.result(),
+            "best_oc": sm.oc_name(best_oc),
+            "per_oc": per_oc,
+            "label_sweep": {"settings_per_oc": args.settings, "reps": 3, "seconds": round(sweep_s, 1)},
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4"])
+    ap.add_argument("--settings", type=int, default=2, help="settings per OC in the label pass")
+    ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--cpu-budget", type=float, default=12.0)
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        ap.error("--warmup must be >= 3")
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_impl(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

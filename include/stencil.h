@@ -245,6 +245,14 @@ int stencil_slab_range(int64_t nz_global, int rank, int nranks, int64_t *z_begin
 /* Thread-local message of the last error (empty string if none). */
 const char *stencil_last_error(void);
 
+/* Kernel timing: with enable = 1, stencil_run brackets every sweep-kernel
+ * launch with CUDA events on the plan's stream; stencil_plan_kernel_time then
+ * synchronises the last event and returns (and resets) the summed device time
+ * of those launches and their count. Used by the benchmark's roofline figure
+ * (achieved bytes / average launch duration). */
+int stencil_plan_set_timing(stencil_plan_t plan, int enable);
+int stencil_plan_kernel_time(stencil_plan_t plan, double *kernel_ms, int64_t *launches);
+
 /* Number of kernels this library launched in this process so far (for the
  * benchmark's gpu_launches count). */
 uint64_t stencil_launch_count(void);

@@ -92,6 +92,9 @@ _SIGS = {
     "stencil_plan_set_comm": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int, ctypes.c_int]),
     "stencil_slab_range": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int, ctypes.c_int,
                                           ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64)]),
+    "stencil_plan_set_timing": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int]),
+    "stencil_plan_kernel_time": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_double),
+                                                ctypes.POINTER(ctypes.c_int64)]),
     "stencil_last_error": (ctypes.c_char_p, []),
     "stencil_launch_count": (ctypes.c_uint64, []),
     "stencil_abi_version": (ctypes.c_int, []),
@@ -321,6 +324,15 @@ class Plan:
             "best_params": [bp[i].to_dict() for i in range(NUM_OC)],
             "best_oc": int(best.value),
         }
+
+    def set_timing(self, enable: bool) -> None:
+        _check(lib().stencil_plan_set_timing(self._h, int(bool(enable))))
+
+    def kernel_time(self) -> Tuple[float, int]:
+        """(summed device ms of the sweep-kernel launches since the last call, launches)."""
+        ms, n = ctypes.c_double(), ctypes.c_int64()
+        _check(lib().stencil_plan_kernel_time(self._h, ctypes.byref(ms), ctypes.byref(n)))
+        return float(ms.value), int(n.value)
 
     def set_comm(self, uid: bytes, rank: int, nranks: int) -> None:
         buf = (ctypes.c_uint8 * 128).from_buffer_copy(uid)

@@ -418,9 +418,23 @@ static int launch_sweep(stencil_plan_s* P, const Variant& v, const Kernel& k, co
   (void)nargs;
   if (gy > 65535 || gz > 65535) SM_FAIL(STENCIL_E_OC_INFEASIBLE, "grid too large for this tile setting");
   const int smem = v.smem_bytes(P->pat, elem);
+  if (P->timing) {
+    if (P->ev_pool.size() < P->ev_used + 2) {
+      for (int i = 0; i < 64; ++i) {
+        cudaEvent_t e;
+        SM_CUDA(cudaEventCreate(&e));
+        P->ev_pool.push_back(e);
+      }
+    }
+    SM_CUDA(cudaEventRecord(P->ev_pool[P->ev_used], P->stream));
+  }
   CUresult r = d->launchKernel(k.fn, gx, gy, gz, bx, by, 1, smem, (CUstream)P->stream, args, nullptr);
   g_launches.fetch_add(1);
   if (r != CUDA_SUCCESS) SM_FAIL(STENCIL_E_CUDA, "cuLaunchKernel(%s): %s", P->lowered.c_str(), cu_errstr(r));
+  if (P->timing) {
+    SM_CUDA(cudaEventRecord(P->ev_pool[P->ev_used + 1], P->stream));
+    P->ev_used += 2;
+  }
   return STENCIL_OK;
 }
 
@@ -452,6 +466,7 @@ int run_device(stencil_plan_s* P, const void* in, void* out, int steps);
 using namespace smart_rt;
 
 stencil_plan_s::~stencil_plan_s() {
+  for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
   if (h_in_dev) cudaFree(h_in_dev);
   if (h_out_dev) cudaFree(h_out_dev);
   if (h_ws_dev) cudaFree(h_ws_dev);
@@ -638,6 +653,30 @@ int stencil_plan_info(stencil_plan_t P, stencil_plan_info_t* info) {
   for (int k = 0; k < 3; ++k) pts *= (P->vdims[k] - 2 * P->frame[k]);
   info->points = pts;
   snprintf(info->kernel_name, sizeof info->kernel_name, "%s", P->lowered.c_str());
+  return STENCIL_OK;
+}
+
+int stencil_plan_set_timing(stencil_plan_t P, int enable) {
+  clear_error();
+  if (!P) SM_FAIL(STENCIL_E_INVAL, "null plan");
+  P->timing = enable != 0;
+  P->ev_used = 0;
+  return STENCIL_OK;
+}
+
+int stencil_plan_kernel_time(stencil_plan_t P, double* kernel_ms, int64_t* launches) {
+  clear_error();
+  if (!P || !kernel_ms || !launches) SM_FAIL(STENCIL_E_INVAL, "null argument");
+  double tot = 0.0;
+  if (P->ev_used) SM_CUDA(cudaEventSynchronize(P->ev_pool[P->ev_used - 1]));
+  for (size_t i = 0; i + 1 < P->ev_used; i += 2) {
+    float ms = 0.f;
+    SM_CUDA(cudaEventElapsedTime(&ms, P->ev_pool[i], P->ev_pool[i + 1]));
+    tot += ms;
+  }
+  *kernel_ms = tot;
+  *launches = (int64_t)(P->ev_used / 2);
+  P->ev_used = 0;
   return STENCIL_OK;
 }
 

@@ -158,6 +158,11 @@ struct stencil_plan_s {
   void* h_out_dev = nullptr;
   void* h_ws_dev = nullptr;
 
+  // kernel timing (stencil_plan_set_timing)
+  bool timing = false;
+  std::vector<cudaEvent_t> ev_pool;      // pairs: [2i] before, [2i+1] after launch i
+  size_t ev_used = 0;
+
   // multi-GPU
   smart_rt::Comm* comm = nullptr;
 
