@@ -248,6 +248,8 @@ def run_impl(args):
     info0 = base_plan.info
     pts = info0["points"]
     ocs = _ocs_for(name, sm)
+    if args.oc:
+        ocs = [sm.oc_from_name(args.oc)]
     t_sw = time.time()
     if args.settings > 0 and len(ocs) > 1:
         sweep = base_plan.oc_sweep(x, y, steps=steps, settings_per_oc=args.settings, reps=3, seed=args.seed)
@@ -272,6 +274,8 @@ def run_impl(args):
             best_oc, best_t, best_p = oc, t, p
     if best_oc is None:
         best_oc, best_p = ocs[0], None
+    if args.params:
+        best_p = json.loads(args.params)
     if world > 1:   # every rank must run the same OC: take rank 0's label
         obj = [best_oc, best_p]
         dist.broadcast_object_list(obj, src=0)
@@ -388,6 +392,8 @@ def main():
     ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4"])
     ap.add_argument("--settings", type=int, default=2, help="settings per OC in the label pass")
     ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--oc", default="", help="time this OC (skips the label pass); for profiling")
+    ap.add_argument("--params", default="", help="JSON parameter setting for --oc")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")

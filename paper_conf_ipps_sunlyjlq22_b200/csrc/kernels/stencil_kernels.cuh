@@ -572,4 +572,178 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
   }
 }
 
+// ===========================================================================
+// Streaming + temporal blocking: OC ST_TB and its combinations (
+// the AN5D-style pipeline of [15]). A CTA streams one (x,y) tile through TT
+// time steps at once: input planes (tile + TT*extent halo) arrive by TMA;
+// stage s = 1..TT-1 computes plane p - s*ZHI of time step s on the tile
+// expanded by (TT-s)*extent and keeps it in its own shared-memory ring of NZ
+// planes; the last stage writes output plane p - TT*ZHI to global memory.
+// Halos are recomputed redundantly (the paper's "redundantly loading from
+// adjacent blocks"); the frame is re-imposed at every stage. Every ring uses
+// the input plane geometry, so (x,y) has the same offset in all of them.
+// Intermediate stages evaluate one point per thread-iteration (gather); the
+// last stage uses the M x VX register tile (BM/CM) in gather form, or in the
+// retiming (RT) scatter form with its register queue of partial sums.
+// ===========================================================================
+template <class S, int BX, int BY, int VX, int M, bool CM, bool RT, int NS, int TT>
+struct StreamTbCfg {
+  typedef typename S::T T;
+  static constexpr int ALN = (16 / (int)sizeof(T)) > VX ? (16 / (int)sizeof(T)) : VX;
+  static constexpr int XOFF = ((TT * S::XLO + ALN - 1) / ALN) * ALN;
+  static constexpr int LX = ((XOFF + BX + TT * S::XHI + ALN - 1) / ALN) * ALN;
+  static constexpr int LY = BY * M + TT * (S::YLO + S::YHI);
+  static constexpr int PLANE = ((LX * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
+  static constexpr int NIN = S::NZ + NS - 1;          // input ring (stage 0)
+  static constexpr int NMID = S::NZ;                  // ring of each stage 1..TT-1
+  static constexpr int SMEM = (NIN + (TT - 1) * NMID) * PLANE * (int)sizeof(T) + 8 * NIN + 128;
+  static constexpr int THREADS = (BX / VX) * BY;
+};
+
+template <class S, int BX, int BY, int VX, int M, bool CM, bool RT, int NS, int TT>
+__global__ void __launch_bounds__((BX / VX) * BY)
+k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, Grid g, int chunk,
+            const __grid_constant__ TmaDesc tmap) {
+  typedef typename S::T T;
+  typedef StreamTbCfg<S, BX, BY, VX, M, CM, RT, NS, TT> C;
+  constexpr int NZ = S::NZ;
+  static_assert(TT >= 2, "k_stream_tb needs TT >= 2");
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  T* ring0 = reinterpret_cast<T*>(smem_raw);
+  T* mid = ring0 + C::NIN * C::PLANE;                  // stage s ring: mid + (s-1)*NZ*PLANE
+  unsigned long long* bar =
+      reinterpret_cast<unsigned long long*>(smem_raw + (C::NIN + (TT - 1) * C::NMID) * C::PLANE * sizeof(T));
+
+  const int tid = threadIdx.y * (BX / VX) + threadIdx.x;
+  const int xa = (g.cx0 / C::ALN) * C::ALN;
+  const int xb = xa + blockIdx.x * BX;
+  const int yb = g.cy0 + blockIdx.y * BY * M;
+  const int zs = g.cz0 + blockIdx.z * chunk;
+  const int ze = min(zs + chunk, g.cz1);
+  const int pin0 = zs - TT * S::ZLO;                   // first input plane
+  const int nit = (ze - zs) + TT * (NZ - 1);
+  const int X0 = xb - C::XOFF, Y0 = yb - TT * S::YLO;
+
+  auto issue = [&](int it) {
+    const int slot = it % C::NIN;
+    if (tid == 0) {
+      mbar_expect_tx(&bar[slot], C::LX * C::LY * (unsigned)sizeof(T));
+      tma_load_3d(ring0 + slot * C::PLANE, &tmap, &bar[slot], X0, Y0, pin0 + it);
+    }
+  };
+  // plane pointer of stage k (0 = input) holding plane q
+  auto stage_plane = [&](int k, int q) -> T* {
+    const int idx = q - (zs - (TT - k) * S::ZLO);
+    return k == 0 ? ring0 + (idx % C::NIN) * C::PLANE : mid + ((k - 1) * NZ + idx % NZ) * C::PLANE;
+  };
+
+  if (tid == 0) {
+    tma_prefetch_desc(&tmap);
+    for (int s = 0; s < C::NIN; ++s) mbar_init(&bar[s], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+#pragma unroll 1
+  for (int it = 0; it < NS - 1; ++it)
+    if (it < nit) issue(it);
+
+  // stage s (1..TT-1) of iteration it: plane q = p - s*ZHI on region R_s
+  auto mid_stage = [&](int it, int s) {
+    if (it < s * (NZ - 1)) return;
+    const int q = pin0 + it - s * S::ZHI;
+    T* dst = stage_plane(s, q);
+    if (q < 0 || q >= g.nz) return;                   // outside the array: never consumed
+    const T* src[NZ];
+#pragma unroll
+    for (int zi = 0; zi < NZ; ++zi) src[zi] = stage_plane(s - 1, q + zi - S::ZLO);
+    const bool zupd = q >= g.uz0 && q < g.uz1;
+    const int hx0 = (TT - s) * S::XLO, hy0 = (TT - s) * S::YLO;
+    const int RX = BX + hx0 + (TT - s) * S::XHI, RY = BY * M + hy0 + (TT - s) * S::YHI;
+    for (int i = tid; i < RX * RY; i += C::THREADS) {
+      const int gx = xb - hx0 + i % RX, gy = yb - hy0 + i / RX;
+      if (gx < 0 || gx >= g.nx || gy < 0 || gy >= g.ny) continue;
+      const int li = (gy - Y0) * C::LX + (gx - X0);
+      if (!(zupd && gy >= g.uy0 && gy < g.uy1 && gx >= g.ux0 && gx < g.ux1)) {
+        dst[li] = src[S::ZLO][li];                      // frame: value unchanged
+        continue;
+      }
+      T acc = T(0);
+#pragma unroll
+      for (int zi = 0; zi < S::NZ; ++zi)
+#pragma unroll
+        for (int yi = 0; yi < S::NY; ++yi)
+#pragma unroll
+          for (int xi = 0; xi < S::NX; ++xi) {
+            const int id = cidx<S>(zi, yi, xi);
+            if (id >= 0) acc = fma_t(S::coef(id), src[zi][li + (yi - S::YLO) * C::LX + (xi - S::XLO)], acc);
+          }
+      dst[li] = acc;
+    }
+  };
+
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int row0 = TT * S::YLO + (CM ? ty : ty * M);
+  const int col0 = C::XOFF + tx * VX;
+  const int x0 = xb + tx * VX;
+  const int y0 = yb + (CM ? ty : ty * M);
+
+  // one pipeline iteration up to (excluding) the last stage
+  auto front = [&](int it) {
+    if (it + NS - 1 < nit) issue(it + NS - 1);
+    mbar_wait(&bar[it % C::NIN], (unsigned)((it / C::NIN) & 1));
+#pragma unroll 1
+    for (int s = 1; s < TT; ++s) {
+      mid_stage(it, s);
+      __syncthreads();
+    }
+  };
+
+  if constexpr (RT) {
+    T acc[NZ][M][VX];
+#pragma unroll
+    for (int q = 0; q < NZ; ++q) zero_acc<T, VX, M>(acc[q]);
+    // the last stage consumes stage TT-1 plane q = p - (TT-1)*ZHI, produced
+    // from iteration (TT-1)*(NZ-1) on; its index j = it - (TT-1)*(NZ-1).
+    constexpr int J0 = (TT - 1) * (NZ - 1);
+#pragma unroll 1
+    for (int itb = 0; itb < nit; itb += NZ) {
+      static_for<0, NZ>([&](auto ic) {
+        constexpr int U = decltype(ic)::value;
+        const int it = itb + U;
+        if (it < nit) {
+          front(it);
+          if (it >= J0) {
+            // rotation index of this stage-(TT-1) plane: (it - J0) % NZ, kept
+            // compile-time by requiring J0 % NZ handled through U' = (U - J0%NZ)
+            constexpr int UR = ((U - J0 % NZ) % NZ + NZ) % NZ;
+            const int q = pin0 + it - (TT - 1) * S::ZHI;
+            zero_acc<T, VX, M>(acc[UR]);
+            SmemPlane<T, VX, C::LX> pl{stage_plane(TT - 1, q) + row0 * C::LX + col0};
+            run_scatter<S, VX, M, UR>(pl, acc);
+            const int z = q - S::ZHI;
+            if (z >= zs) store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc[(UR + 1) % NZ]);
+          }
+          __syncthreads();
+        }
+      });
+    }
+  } else {
+#pragma unroll 1
+    for (int it = 0; it < nit; ++it) {
+      front(it);
+      if (it >= TT * (NZ - 1)) {
+        const int z = pin0 + it - TT * S::ZHI;
+        T acc[M][VX];
+        zero_acc<T, VX, M>(acc);
+        SmemPlane<T, VX, C::LX> pl[NZ];
+#pragma unroll
+        for (int zi = 0; zi < NZ; ++zi) pl[zi].p = stage_plane(TT - 1, z + zi - S::ZLO) + row0 * C::LX + col0;
+        run_gather<S, VX, M>(pl, acc);
+        store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc);
+      }
+      __syncthreads();
+    }
+  }
+}
+
 }  // namespace smart

@@ -230,8 +230,9 @@ static TmaBox tma_box(const Variant& v, const Pattern& p, int elem) {
     return {ru(xoff + v.bx + v.tt * p.xhi, aln), v.by * v.m + v.tt * (p.ylo + p.yhi),
             v.bz + v.tt * (p.zlo + p.zhi)};
   }
-  const int xoff = ru(p.xlo, aln);
-  return {ru(xoff + v.bx + p.xhi, aln), v.by * v.m + p.ylo + p.yhi, 1};
+  const int t = v.family == FAM_STREAM_TB ? v.tt : 1;   // stream: halo of t time steps
+  const int xoff = ru(t * p.xlo, aln);
+  return {ru(xoff + v.bx + t * p.xhi, aln), v.by * v.m + t * (p.ylo + p.yhi), 1};
 }
 
 static int resolve_variant(stencil_plan_s* P) {
@@ -251,9 +252,6 @@ static int resolve_variant(stencil_plan_s* P) {
     if (fam == FAM_STREAM || fam == FAM_STREAM_TB) { v.by = 1; v.m = 1; }
     else v.bz = 1;
   }
-  if (fam == FAM_STREAM_TB)
-    SM_FAIL(STENCIL_E_OC_INFEASIBLE, "OC %s: streaming + temporal blocking kernel not built yet",
-            oc_name_static(P->oc));
   if (v.vx != 1 && v.vx != 2 && v.vx != 4) SM_FAIL(STENCIL_E_INVAL, "vx must be 1, 2 or 4");
   if (v.vx * elem > 32) SM_FAIL(STENCIL_E_INVAL, "vx*sizeof(T) must be <= 32 bytes");
   if (!pow2(v.bx) || !pow2(v.by) || !pow2(v.bz) || !pow2(v.m) || v.bx < v.vx)
@@ -271,11 +269,15 @@ static int resolve_variant(stencil_plan_s* P) {
             oc_name_static(P->oc), smem);
   // TMA staging when rows are 16-byte multiples and the box fits 256^3
   v.tma = false;
-  if (fam == FAM_TILED || fam == FAM_STREAM) {
+  if (fam == FAM_TILED || fam == FAM_STREAM || fam == FAM_STREAM_TB) {
     const TmaBox b = tma_box(v, P->pat, elem);
     const bool rows_ok = (P->vdims[2] * elem) % 16 == 0;
     v.tma = rows_ok && b.lx <= 256 && b.ly <= 256 && b.lz <= 256 && getenv("STENCIL_NO_TMA") == nullptr;
   }
+  if (fam == FAM_STREAM_TB && !v.tma)
+    SM_FAIL(STENCIL_E_OC_INFEASIBLE, "OC %s needs TMA staging (rows of 16-byte multiples, box <= 256)",
+            oc_name_static(P->oc));
+  if (fam == FAM_STREAM_TB && v.tt < 2) v.family = FAM_STREAM;
   v.chunk = p.stream_chunk;
   P->var = v;
   return STENCIL_OK;
@@ -441,6 +443,7 @@ static int launch_sweep(stencil_plan_s* P, const Variant& v, const Kernel& k, co
 static int get_tb_rem_kernel(stencil_plan_s* P, int tt, Variant* vout, Kernel* kout) {
   Variant v = P->var;
   v.tt = tt;
+  if (v.family == FAM_STREAM_TB && tt == 1) v.family = FAM_STREAM;   // remainder of one step: plain ST
   const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
   if (v.family == FAM_TILED && v.tma) {
     const TmaBox b = tma_box(v, P->pat, elem);
@@ -593,7 +596,22 @@ int stencil_plan_create(stencil_plan_t* plan, int ndim, const int64_t* dims, int
   merge_params(params, &P->params);
   SM_TRY(build_pattern(P.get()));
   build_view(P.get(), family_of(oc, P->params.smem));
-  SM_TRY(resolve_variant(P.get()));
+  // Default tiles shrink until the shared-memory footprint fits (high-order
+  // stencils under TB need smaller tiles); user-given fields are kept.
+  const bool user_bz = params && params->bz, user_by = params && params->by, user_bx = params && params->bx;
+  for (int attempt = 0;; ++attempt) {
+    const int rc = resolve_variant(P.get());
+    if (rc != STENCIL_E_OC_INFEASIBLE || attempt > 12) {
+      if (rc != STENCIL_OK) return rc;
+      break;
+    }
+    stencil_params_t& q = P->params;
+    if (!user_bz && q.bz > 1) q.bz /= 2;
+    else if (!user_by && q.by > 1 && (q.bx / std::max(q.vx, 1)) * (q.by / 2) >= 32) q.by /= 2;
+    else if (!user_bx && q.bx > 8 * q.vx) q.bx /= 2;
+    else return rc;
+  }
+  clear_error();
   P->src = generate_source(P->pat, P->dtype, P->var);
   // kernel specialisation (host-only; module load is deferred to first use)
   SM_TRY(compile_variant(P->pat, P->dtype, P->var, &P->lowered, &P->cubin));

@@ -109,8 +109,8 @@ std::string Variant::name_expr(const char* desc) const {
                rt ? "true" : "false", ns, tf);
       break;
     default:
-      snprintf(b, sizeof b, "smart::k_stream_tb<%s, %d, %d, %d, %d, %s, %s, %d, %d, %s>", desc, bx, by, vx,
-               m, cmf, rt ? "true" : "false", ns, tt, tf);
+      snprintf(b, sizeof b, "smart::k_stream_tb<%s, %d, %d, %d, %d, %s, %s, %d, %d>", desc, bx, by, vx, m,
+               cmf, rt ? "true" : "false", ns, tt);
       break;
   }
   return b;
@@ -144,6 +144,15 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     const int nz = p.zlo + p.zhi + 1;
     const int nring = (rt ? 1 : nz) + ns - 1;
     return nring * plane * elem + 8 * nring + 128;
+  }
+  if (family == FAM_STREAM_TB) {   // mirrors StreamTbCfg
+    const int xoff = roundup(tt * p.xlo, aln);
+    const int lx = roundup(xoff + bx + tt * p.xhi, aln);
+    const int ly = by * m + tt * (p.ylo + p.yhi);
+    const int plane = roundup(lx * ly * elem, 128) / elem;
+    const int nz = p.zlo + p.zhi + 1;
+    const int nin = nz + ns - 1;
+    return (nin + (tt - 1) * nz) * plane * elem + 8 * nin + 128;
   }
   return 0;
 }
