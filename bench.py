@@ -205,13 +205,26 @@ def run_reference(args):
     return 0
 
 
-def _traffic_from_profiles(kernel_name: str):
+def kernel_key(config: str, lowered: str) -> str:
+    """'C2:k_stream<16,8,1,8,0,0,1,1>' from a mangled NVRTC kernel name."""
+    import re
+    m = re.match(r"_ZN5smart(\d+)", lowered)
+    if not m:
+        return f"{config}:{lowered}"
+    n = int(m.group(1))
+    start = m.end()
+    name = lowered[start:start + n]
+    args = re.findall(r"L[ib](\d+)E", lowered[start + n:])
+    return f"{config}:{name}<{','.join(args)}>"
+
+
+def _traffic_from_profiles(key: str):
+    """dram read+write bytes per launch from a committed `ncu --set full` capture."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if not os.path.exists(p):
         return None
     try:
-        d = json.load(open(p))
-        e = d.get(kernel_name)
+        e = json.load(open(p)).get(key)
         return float(e["dram_bytes_per_launch"]) if e else None
     except Exception:
         return None
@@ -319,8 +332,10 @@ def run_impl(args):
     avg_launch_ms = kern_ms / max(kern_n, 1)
     achieved = bytes_per_launch / (avg_launch_ms * 1e-3) / 1e9
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(achieved / peak, 4), "traffic": _traffic_from_profiles(pinfo["kernel_name"]),
-                "peak_kind": peak_kind, "kernel": pinfo["kernel_name"][:100], "launch_ms": round(avg_launch_ms, 4),
+                "frac": round(achieved / peak, 4),
+                "traffic": _traffic_from_profiles(kernel_key(name, pinfo["kernel_name"])),
+                "peak_kind": peak_kind, "kernel": kernel_key(name, pinfo["kernel_name"]),
+                "launch_ms": round(avg_launch_ms, 4),
                 "kernel_share_of_step": round(kern_ms / max(total_ms, 1e-9), 4),
                 "bytes_per_launch": bytes_per_launch, "time_steps_per_launch": T,
                 "frac_of_spec_8tbs": round(achieved / HBM_SPEC_GBS, 4)}
