@@ -203,13 +203,15 @@ struct GlobalPlane {                  // global memory through the read-only pat
 //              partial sums of output plane p - (zi - ZLO), kept in
 //              acc[(U + NZ - zi) % NZ] (a register queue rotated at compile time).
 // ---------------------------------------------------------------------------
-template <class S, int VX, int M, class L>
-__device__ __forceinline__ void run_gather(const L (&pl)[S::NZ], typename S::T (&acc)[M][VX]) {
+// O: the op table (S itself for the main table, S::Mid for the intermediate
+// fused steps of k_stream_tb).
+template <class S, class O, int VX, int M, class L>
+__device__ __forceinline__ void run_gather_ops(const L (&pl)[S::NZ], typename S::T (&acc)[M][VX]) {
   typedef typename S::T T;
   T w[VX];
 #pragma unroll
-  for (int i = 0; i < S::NOPS; ++i) {
-    const unsigned op = S::op(i);
+  for (int i = 0; i < O::NOPS; ++i) {
+    const unsigned op = O::op(i);
     if (!(op >> 31)) {
       pl[op & 15].get(int((op >> 4) & 255) - 128, int((op >> 12) & 15) - 8, w);
     } else {
@@ -217,6 +219,11 @@ __device__ __forceinline__ void run_gather(const L (&pl)[S::NZ], typename S::T (
       a = fma_t(S::coef(op & 1023), w[(op >> 10) & 3], a);
     }
   }
+}
+
+template <class S, int VX, int M, class L>
+__device__ __forceinline__ void run_gather(const L (&pl)[S::NZ], typename S::T (&acc)[M][VX]) {
+  run_gather_ops<S, S, VX, M>(pl, acc);
 }
 
 template <class S, int VX, int M, int U, class L>
@@ -582,9 +589,10 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
 // Halos are recomputed redundantly (the paper's "redundantly loading from
 // adjacent blocks"); the frame is re-imposed at every stage. Every ring uses
 // the input plane geometry, so (x,y) has the same offset in all of them.
-// Intermediate stages evaluate one point per thread-iteration (gather); the
-// last stage uses the M x VX register tile (BM/CM) in gather form, or in the
-// retiming (RT) scatter form with its register queue of partial sums.
+// Intermediate stages are computed in VX x MI register tiles (gather, op
+// table S::Mid); the last stage uses the M x VX register tile (BM/CM) in
+// gather form, or in the retiming (RT) scatter form with its register queue of
+// partial sums.
 // ===========================================================================
 template <class S, int BX, int BY, int VX, int M, bool CM, bool RT, int NS, int TT>
 struct StreamTbCfg {
@@ -596,7 +604,12 @@ struct StreamTbCfg {
   static constexpr int PLANE = ((LX * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
   static constexpr int NIN = S::NZ + NS - 1;          // input ring (stage 0)
   static constexpr int NMID = S::NZ;                  // ring of each stage 1..TT-1
-  static constexpr int SMEM = (NIN + (TT - 1) * NMID) * PLANE * (int)sizeof(T) + 8 * NIN + 128;
+  static constexpr int MI = S::MI;                    // rows of an intermediate-stage thread tile
+  // intermediate tiles are rounded to VX x MI, so their (discarded) edge values
+  // read up to VX elements before a plane and MI rows after it: pad both ends
+  static constexpr int PADF = 128 / (int)sizeof(T);
+  static constexpr int PADB = ((MI * LX + ALN) * (int)sizeof(T) + 127) / 128 * 128 / (int)sizeof(T);
+  static constexpr int SMEM = (PADF + (NIN + (TT - 1) * NMID) * PLANE + PADB) * (int)sizeof(T) + 8 * NIN + 128;
   static constexpr int THREADS = (BX / VX) * BY;
 };
 
@@ -607,12 +620,13 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
   typedef typename S::T T;
   typedef StreamTbCfg<S, BX, BY, VX, M, CM, RT, NS, TT> C;
   constexpr int NZ = S::NZ;
+  constexpr int MI = C::MI;
   static_assert(TT >= 2, "k_stream_tb needs TT >= 2");
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  T* ring0 = reinterpret_cast<T*>(smem_raw);
+  T* ring0 = reinterpret_cast<T*>(smem_raw) + C::PADF;
   T* mid = ring0 + C::NIN * C::PLANE;                  // stage s ring: mid + (s-1)*NZ*PLANE
-  unsigned long long* bar =
-      reinterpret_cast<unsigned long long*>(smem_raw + (C::NIN + (TT - 1) * C::NMID) * C::PLANE * sizeof(T));
+  unsigned long long* bar = reinterpret_cast<unsigned long long*>(
+      smem_raw + (C::PADF + (C::NIN + (TT - 1) * C::NMID) * C::PLANE + C::PADB) * sizeof(T));
 
   const int tid = threadIdx.y * (BX / VX) + threadIdx.x;
   const int xa = (g.cx0 / C::ALN) * C::ALN;
@@ -647,37 +661,55 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
   for (int it = 0; it < NS - 1; ++it)
     if (it < nit) issue(it);
 
-  // stage s (1..TT-1) of iteration it: plane q = p - s*ZHI on region R_s
-  auto mid_stage = [&](int it, int s) {
+  // Intermediate fused step s (1..TT-1) of iteration it: plane q = p - s*ZHI
+  // on region R_s (tile expanded by (TT-s)*extent), computed in VX x MI
+  // register tiles with the S::Mid op table; values outside R_s, the array or
+  // the update box are masked / copied (frame re-imposed).
+  auto mid_stage = [&](int it, auto sc) {
+    constexpr int s = decltype(sc)::value;
+    constexpr int HX0 = (TT - s) * S::XLO, HX1 = (TT - s) * S::XHI;
+    constexpr int HY0 = (TT - s) * S::YLO, HY1 = (TT - s) * S::YHI;
+    constexpr int TXL = ((HX0 + VX - 1) / VX) * VX;
+    constexpr int NTX = (TXL + BX + HX1 + VX - 1) / VX;
+    constexpr int RY = BY * M + HY0 + HY1;
+    constexpr int NTY = (RY + MI - 1) / MI;
     if (it < s * (NZ - 1)) return;
     const int q = pin0 + it - s * S::ZHI;
-    T* dst = stage_plane(s, q);
     if (q < 0 || q >= g.nz) return;                   // outside the array: never consumed
+    T* dst = stage_plane(s, q);
+    const T* ctr = stage_plane(s - 1, q);
     const T* src[NZ];
 #pragma unroll
     for (int zi = 0; zi < NZ; ++zi) src[zi] = stage_plane(s - 1, q + zi - S::ZLO);
     const bool zupd = q >= g.uz0 && q < g.uz1;
-    const int hx0 = (TT - s) * S::XLO, hy0 = (TT - s) * S::YLO;
-    const int RX = BX + hx0 + (TT - s) * S::XHI, RY = BY * M + hy0 + (TT - s) * S::YHI;
-    for (int i = tid; i < RX * RY; i += C::THREADS) {
-      const int gx = xb - hx0 + i % RX, gy = yb - hy0 + i / RX;
-      if (gx < 0 || gx >= g.nx || gy < 0 || gy >= g.ny) continue;
-      const int li = (gy - Y0) * C::LX + (gx - X0);
-      if (!(zupd && gy >= g.uy0 && gy < g.uy1 && gx >= g.ux0 && gx < g.ux1)) {
-        dst[li] = src[S::ZLO][li];                      // frame: value unchanged
-        continue;
-      }
-      T acc = T(0);
+    const int rx0 = xb - HX0, rx1 = xb + BX + HX1, ry0 = yb - HY0, ry1 = yb + BY * M + HY1;
+    for (int t = tid; t < NTX * NTY; t += C::THREADS) {
+      const int gx0 = xb - TXL + (t % NTX) * VX, gy0 = ry0 + (t / NTX) * MI;
+      const int lbase = (gy0 - Y0) * C::LX + (gx0 - X0);
+      T acc[MI][VX];
+      zero_acc<T, VX, MI>(acc);
+      SmemPlane<T, VX, C::LX> pl[NZ];
 #pragma unroll
-      for (int zi = 0; zi < S::NZ; ++zi)
+      for (int zi = 0; zi < NZ; ++zi) pl[zi].p = src[zi] + lbase;
+      run_gather_ops<S, typename S::Mid, VX, MI>(pl, acc);
 #pragma unroll
-        for (int yi = 0; yi < S::NY; ++yi)
+      for (int m = 0; m < MI; ++m) {
+        const int gy = gy0 + m;
+        if (gy >= ry1 || gy < 0 || gy >= g.ny) continue;
+        const bool rowupd = zupd && gy >= g.uy0 && gy < g.uy1;
+        const int li = lbase + m * C::LX;
+        if (rowupd && gx0 >= rx0 && gx0 + VX <= rx1 && gx0 >= g.ux0 && gx0 + VX <= g.ux1) {
+          stg_vec<T, VX>(dst + li, acc[m]);             // whole vector interior
+        } else {
 #pragma unroll
-          for (int xi = 0; xi < S::NX; ++xi) {
-            const int id = cidx<S>(zi, yi, xi);
-            if (id >= 0) acc = fma_t(S::coef(id), src[zi][li + (yi - S::YLO) * C::LX + (xi - S::XLO)], acc);
+          for (int v = 0; v < VX; ++v) {
+            const int gx = gx0 + v;
+            if (gx < rx0 || gx >= rx1 || gx < 0 || gx >= g.nx) continue;
+            const bool upd = rowupd && gx >= g.ux0 && gx < g.ux1;
+            dst[li + v] = upd ? acc[m][v] : ctr[li + v];
           }
-      dst[li] = acc;
+        }
+      }
     }
   };
 
@@ -691,11 +723,10 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
   auto front = [&](int it) {
     if (it + NS - 1 < nit) issue(it + NS - 1);
     mbar_wait(&bar[it % C::NIN], (unsigned)((it / C::NIN) & 1));
-#pragma unroll 1
-    for (int s = 1; s < TT; ++s) {
-      mid_stage(it, s);
+    static_for<1, TT>([&](auto sc) {
+      mid_stage(it, sc);
       __syncthreads();
-    }
+    });
   };
 
   if constexpr (RT) {
@@ -706,26 +737,25 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
     // from iteration (TT-1)*(NZ-1) on; its index j = it - (TT-1)*(NZ-1).
     constexpr int J0 = (TT - 1) * (NZ - 1);
 #pragma unroll 1
-    for (int itb = 0; itb < nit; itb += NZ) {
-      static_for<0, NZ>([&](auto ic) {
-        constexpr int U = decltype(ic)::value;
-        const int it = itb + U;
-        if (it < nit) {
-          front(it);
-          if (it >= J0) {
-            // rotation index of this stage-(TT-1) plane: (it - J0) % NZ, kept
-            // compile-time by requiring J0 % NZ handled through U' = (U - J0%NZ)
-            constexpr int UR = ((U - J0 % NZ) % NZ + NZ) % NZ;
-            const int q = pin0 + it - (TT - 1) * S::ZHI;
+    for (int it = 0; it < nit; ++it) {
+      front(it);
+      if (it >= J0) {
+        // rotation index of this stage-(TT-1) plane; each branch below uses
+        // compile-time queue indices, so the partial sums stay in registers
+        const int ur = (it - J0) % NZ;
+        const int q = pin0 + it - (TT - 1) * S::ZHI;
+        SmemPlane<T, VX, C::LX> pl{stage_plane(TT - 1, q) + row0 * C::LX + col0};
+        const int z = q - S::ZHI;
+        static_for<0, NZ>([&](auto ic) {
+          constexpr int UR = decltype(ic)::value;
+          if (ur == UR) {
             zero_acc<T, VX, M>(acc[UR]);
-            SmemPlane<T, VX, C::LX> pl{stage_plane(TT - 1, q) + row0 * C::LX + col0};
             run_scatter<S, VX, M, UR>(pl, acc);
-            const int z = q - S::ZHI;
             if (z >= zs) store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc[(UR + 1) % NZ]);
           }
-          __syncthreads();
-        }
-      });
+        });
+      }
+      __syncthreads();
     }
   } else {
 #pragma unroll 1

@@ -125,6 +125,9 @@ int Variant::threads() const {
 
 static int roundup(int a, int b) { return (a + b - 1) / b * b; }
 
+// rows of an intermediate-stage thread tile in k_stream_tb (S::MI)
+static constexpr int kMidRows = 2;
+
 // Mirrors TiledCfg / StreamCfg of stencil_kernels.cuh.
 int Variant::smem_bytes(const Pattern& p, int elem) const {
   const int aln = std::max(16 / elem, vx);
@@ -152,7 +155,9 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     const int plane = roundup(lx * ly * elem, 128) / elem;
     const int nz = p.zlo + p.zhi + 1;
     const int nin = nz + ns - 1;
-    return (nin + (tt - 1) * nz) * plane * elem + 8 * nin + 128;
+    const int padf = 128 / elem;
+    const int padb = roundup((kMidRows * lx + aln) * elem, 128) / elem;
+    return (padf + (nin + (tt - 1) * nz) * plane + padb) * elem + 8 * nin + 128;
   }
   return 0;
 }
@@ -253,7 +258,20 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   for (size_t i = 0; i < ops.size(); ++i) o << ops[i] << "u" << (i + 1 < ops.size() ? "," : "");
   if (ops.empty()) o << "0u";
   o << "};\n";
+  std::vector<uint32_t> mops;
+  if (v.family == FAM_STREAM_TB) {     // intermediate fused steps: gather, VX x kMidRows tiles
+    Variant vm = v;
+    vm.family = FAM_STREAM; vm.rt = false; vm.cm = false; vm.m = kMidRows;
+    mops = encode_ops(pat, vm);
+  }
+  o << "__device__ constexpr unsigned g_mops[" << std::max<size_t>(mops.size(), 1) << "] = {";
+  for (size_t i = 0; i < mops.size(); ++i) o << mops[i] << "u" << (i + 1 < mops.size() ? "," : "");
+  if (mops.empty()) o << "0u";
+  o << "};\n";
   o << "struct S {\n  typedef " << T << " T;\n";
+  o << "  static constexpr int MI = " << kMidRows << ";\n";
+  o << "  struct Mid {\n    static constexpr int NOPS = " << mops.size() << ";\n"
+    << "    static __device__ __forceinline__ constexpr unsigned op(int i) { return g_mops[i]; }\n  };\n";
   o << "  static constexpr int NNZ = " << pat.nnz << ", ZLO = " << pat.zlo << ", ZHI = " << pat.zhi
     << ", YLO = " << pat.ylo << ", YHI = " << pat.yhi << ", XLO = " << pat.xlo << ", XHI = " << pat.xhi
     << ", NZ = " << NZ << ", NY = " << NY << ", NX = " << NX << ";\n";
