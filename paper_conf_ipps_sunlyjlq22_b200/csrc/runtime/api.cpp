@@ -156,7 +156,7 @@ static void sample_params(uint32_t oc, int ndim, int dtype, uint64_t seed, int k
   if (!st && !tb) { const int s[] = {0, 1}; p->smem = pick(h, s); }
   if (merge) { const int s[] = {2, 4, 8}; p->merge = pick(h, s); }
   if (tb) { const int s[] = {2, 4}; p->tb_steps = pick(h, s); }
-  if (oc & STENCIL_OC_PR) { const int s[] = {2, 4}; p->pr_stages = pick(h, s); }
+  if (oc & STENCIL_OC_PR) { const int s[] = {2, 3, 4}; p->pr_stages = pick(h, s); }   // enum
   const int fam = family_of(oc, p->smem);
   if (fam == FAM_NAIVE) {
     const int sx[] = {32, 64, 128}, sy[] = {1, 2, 4, 8};

@@ -94,9 +94,10 @@ def test_sample_params_deterministic_and_pow2():
             a = sm.sample_params(oc, 3, "f64", 1234, k)
             b = sm.sample_params(oc, 3, "f64", 1234, k)
             assert a == b
-            for key in ("bx", "by", "bz", "vx", "merge", "tb_steps", "pr_stages"):
+            for key in ("bx", "by", "bz", "vx", "merge", "tb_steps"):   # numeric: powers of two
                 v = a[key]
                 assert v > 0 and (v & (v - 1)) == 0, (oc, k, key, v)
+            assert a["pr_stages"] in (1, 2, 3, 4)     # enumeration type, numbered from 1
             assert a["smem"] in (0, 1)
             if not oc & (sm.OC_BM | sm.OC_CM):
                 assert a["merge"] == 1
