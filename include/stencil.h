@@ -226,14 +226,39 @@ int stencil_fill_field(void *dev_ptr, stencil_dtype_t dtype, int ndim, const int
 /* Fill id[128] with a fresh NCCL unique id (call on rank 0, broadcast it). */
 int stencil_nccl_unique_id(uint8_t *id);
 
-/* Attach the plan to a communicator of `nranks` ranks. The plan's grid becomes
- * rank `rank`'s slab: dims[0] local planes of a global grid whose depth is the
- * sum over ranks; the frame exists only at the global faces. Buffers passed to
- * stencil_run then hold only the local slab; halo planes are exchanged with
- * ranks +-1 every step (every T steps for TB) with ncclSend/ncclRecv on the
- * plan's stream, overlapped with the interior sweep. Collective: all ranks call
- * it with the same id. */
+/* Attach the plan (3-D only) to a communicator of `nranks` ranks. The plan's
+ * grid becomes rank `rank`'s slab of a global grid whose depth is the sum of
+ * the ranks' dims[0] (ranks ordered along z); the frame exists only at the
+ * global z faces. Device buffers passed to stencil_run (and the workspace)
+ * then hold dims[0] + 2G planes: G ghost planes, the dims[0] owned planes,
+ * G ghost planes (G = stencil_plan_ghost_planes(plan) = 4*order; dims[0] must
+ * be >= 2G). Each launch computes the edge planes first, exchanges the halo
+ * planes with ranks +-1 (ncclSend/ncclRecv on a comm stream: T*extent planes
+ * every T fused steps) and computes the interior meanwhile; at the start of
+ * stencil_run the ghost planes of `in` are overwritten with the neighbours'
+ * owned planes. Collective: all ranks call it with the same id; tb_steps <= 4. */
 int stencil_plan_set_comm(stencil_plan_t plan, const uint8_t *id, int rank, int nranks);
+
+/* Single-device test form of the decomposition: link `nranks` plans of one
+ * process (rank k = plans[k], same stencil/OC/dtype/plane shape) as slabs of one
+ * global grid; halos move by cudaMemcpyAsync between their buffers, with the
+ * same schedule as the NCCL path. Run them with stencil_run_group. */
+int stencil_plans_link_loopback(stencil_plan_t *plans, int nranks);
+
+/* Advance a loopback group (or one plan: nplans = 1) by `steps` steps:
+ * ins[k] -> outs[k] for every slab k. Same semantics as stencil_run. */
+int stencil_run_group(stencil_plan_t *plans, int nplans, const void *const *ins, void *const *outs,
+                      int steps);
+
+/* G, the ghost planes on each side of the plan's slab (0 without a communicator). */
+int stencil_plan_ghost_planes(stencil_plan_t plan);
+
+/* Host-only halo layout of one exchange (for tests and tools): for a slab of n
+ * owned planes stored at [G, G+n) whose stencil reaches zlo_g planes below and
+ * zhi_g above, writes out[8] = {recv_lo_begin, recv_lo_count, send_lo_begin,
+ * send_lo_count, send_hi_begin, send_hi_count, recv_hi_begin, recv_hi_count}
+ * in local plane indices (lo = rank-1, hi = rank+1; counts 0 at global faces). */
+int stencil_slab_halo(int ghost, int64_t n, int zlo_g, int zhi_g, int rank, int nranks, int64_t *out);
 
 /* Slab layout of `rank` among `nranks` for a global depth nz_global: writes
  * {z_begin, z_end} of the rank's slab (near-equal split). Host only. */

@@ -92,6 +92,13 @@ _SIGS = {
     "stencil_plan_set_comm": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int, ctypes.c_int]),
     "stencil_slab_range": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int, ctypes.c_int,
                                           ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64)]),
+    "stencil_plans_link_loopback": (ctypes.c_int, [ctypes.POINTER(ctypes.c_void_p), ctypes.c_int]),
+    "stencil_run_group": (ctypes.c_int, [ctypes.POINTER(ctypes.c_void_p), ctypes.c_int,
+                                         ctypes.POINTER(ctypes.c_void_p), ctypes.POINTER(ctypes.c_void_p),
+                                         ctypes.c_int]),
+    "stencil_plan_ghost_planes": (ctypes.c_int, [ctypes.c_void_p]),
+    "stencil_slab_halo": (ctypes.c_int, [ctypes.c_int, ctypes.c_int64, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                         ctypes.c_int, ctypes.POINTER(ctypes.c_int64)]),
     "stencil_plan_set_timing": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int]),
     "stencil_plan_kernel_time": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_double),
                                                 ctypes.POINTER(ctypes.c_int64)]),
@@ -177,6 +184,33 @@ def slab_range(nz_global: int, rank: int, nranks: int) -> Tuple[int, int]:
     a, b = ctypes.c_int64(), ctypes.c_int64()
     _check(lib().stencil_slab_range(nz_global, rank, nranks, ctypes.byref(a), ctypes.byref(b)))
     return int(a.value), int(b.value)
+
+
+def slab_halo(ghost: int, n: int, zlo_g: int, zhi_g: int, rank: int, nranks: int) -> Dict[str, Tuple[int, int]]:
+    """Halo plane ranges of one exchange: {'recv_lo': (begin, count), 'send_lo', 'send_hi', 'recv_hi'}."""
+    out = (ctypes.c_int64 * 8)()
+    _check(lib().stencil_slab_halo(ghost, n, zlo_g, zhi_g, rank, nranks, out))
+    v = [int(x) for x in out]
+    return {"recv_lo": (v[0], v[1]), "send_lo": (v[2], v[3]), "send_hi": (v[4], v[5]), "recv_hi": (v[6], v[7])}
+
+
+def link_loopback(plans: Sequence["Plan"]) -> None:
+    """Link plans as the z-slabs (rank order) of one grid on this device."""
+    arr = (ctypes.c_void_p * len(plans))(*[p._h.value for p in plans])
+    _check(lib().stencil_plans_link_loopback(arr, len(plans)))
+
+
+def run_group(plans: Sequence["Plan"], ins, outs, steps: int, stream=None) -> None:
+    L = lib()
+    for p, t in zip(plans, ins):
+        p._check_tensor(t)
+        if steps >= 2:
+            p._ensure_ws(t.device)
+        _check(L.stencil_plan_set_stream(p._h, ctypes.c_void_p(_stream_ptr(stream))))
+    hp = (ctypes.c_void_p * len(plans))(*[p._h.value for p in plans])
+    hi = (ctypes.c_void_p * len(plans))(*[t.data_ptr() for t in ins])
+    ho = (ctypes.c_void_p * len(plans))(*[t.data_ptr() for t in outs])
+    _check(L.stencil_run_group(hp, len(plans), hi, ho, int(steps)))
 
 
 def nccl_unique_id() -> bytes:
@@ -280,10 +314,21 @@ class Plan:
             _check(lib().stencil_plan_set_workspace(self._h, ctypes.c_void_p(self._ws.data_ptr()),
                                                     self.workspace_bytes()))
 
+    @property
+    def ghost(self) -> int:
+        """Ghost planes on each side of the slab (0 without a communicator)."""
+        return int(lib().stencil_plan_ghost_planes(self._h))
+
+    @property
+    def array_shape(self) -> Tuple[int, ...]:
+        """Shape of the device buffers: dims, plus 2*ghost planes along z for a slab."""
+        g = self.ghost
+        return (self.dims[0] + 2 * g,) + self.dims[1:]
+
     def _check_tensor(self, t):
-        if not (t.is_cuda and t.is_contiguous() and t.dtype == self.torch_dtype
-                and tuple(t.shape) == self.dims):
-            raise ValueError(f"expected a contiguous CUDA {self.torch_dtype} tensor of shape {self.dims}")
+        shape = self.array_shape
+        if not (t.is_cuda and t.is_contiguous() and t.dtype == self.torch_dtype and tuple(t.shape) == shape):
+            raise ValueError(f"expected a contiguous CUDA {self.torch_dtype} tensor of shape {shape}")
 
     # -- sweeps
     def run(self, inp, out, steps: int, stream=None) -> None:

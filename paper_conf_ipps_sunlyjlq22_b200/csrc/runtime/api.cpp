@@ -321,6 +321,13 @@ static GridArg make_grid(const stencil_plan_s* P, int elem_vx) {
   g.uy0 = P->frame[1]; g.uy1 = g.ny - P->frame[1];
   g.ux0 = P->frame[2]; g.ux1 = g.nx - P->frame[2];
   g.cz0 = g.uz0; g.cz1 = g.uz1; g.cy0 = g.uy0; g.cy1 = g.uy1; g.cx0 = g.ux0; g.cx1 = g.ux1;
+  if (P->comm) {   // slab: frame only at the global z faces; compute the owned planes
+    const int G = P->ghost, n = (int)P->dims[0], r = P->frame[0];
+    g.uz0 = P->comm->rank == 0 ? G + r : 0;
+    g.uz1 = P->comm->rank == P->comm->nranks - 1 ? G + n - r : g.nz;
+    g.cz0 = std::max(G, g.uz0);
+    g.cz1 = std::min(G + n, g.uz1);
+  }
   g.vec_ok = (g.nx % elem_vx) == 0;
   return g;
 }
@@ -483,42 +490,160 @@ stencil_plan_s::~stencil_plan_s() {
 
 namespace smart_rt {
 
-int run_device(stencil_plan_s* P, const void* in, void* out, int steps) {
-  const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
-  const size_t bytes = (size_t)P->vdims[0] * P->vdims[1] * P->vdims[2] * elem;
-  if (!in || !out) SM_FAIL(STENCIL_E_INVAL, "null grid pointer");
-  if (in == out) SM_FAIL(STENCIL_E_INVAL, "in and out must be distinct buffers");
+// Halo exchange into buffer bufs[k] of every local plan k (a7). NCCL: the
+// plan's comm stream waits for the edge planes, then grouped send/recv with
+// ranks +-1. LOOPBACK: each slab pulls its ghost planes from its neighbours'
+// buffers with cudaMemcpyAsync after their edge planes are written.
+static int exchange(const std::vector<stencil_plan_s*>& Ps, const std::vector<void*>& bufs, int tl) {
+  for (size_t k = 0; k < Ps.size(); ++k) {
+    stencil_plan_s* P = Ps[k];
+    Comm* c = P->comm;
+    if (c->transport == TR_NCCL) {
+      SM_CUDA(cudaStreamWaitEvent(c->stream, c->ev_edge, 0));
+      SM_TRY(comm_exchange_nccl(P, bufs[k], tl));
+    } else {
+      const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+      const size_t pb = (size_t)P->vdims[1] * P->vdims[2] * elem;
+      int64_t h[8];
+      slab_halo(P->ghost, (int)P->dims[0], tl * P->pat.zlo, tl * P->pat.zhi, c->rank, c->nranks, h);
+      SM_CUDA(cudaStreamWaitEvent(c->stream, c->ev_edge, 0));
+      if (h[1]) {   // lower ghosts <- rank-1's last zlo_g owned planes
+        stencil_plan_s* Q = c->peers[c->rank - 1];
+        int64_t hq[8];
+        slab_halo(Q->ghost, (int)Q->dims[0], tl * Q->pat.zlo, tl * Q->pat.zhi, c->rank - 1, c->nranks, hq);
+        SM_CUDA(cudaStreamWaitEvent(c->stream, Q->comm->ev_edge, 0));
+        SM_CUDA(cudaMemcpyAsync((char*)bufs[k] + h[0] * pb, (const char*)bufs[k - 1] + hq[4] * pb, h[1] * pb,
+                                cudaMemcpyDeviceToDevice, c->stream));
+      }
+      if (h[7]) {   // upper ghosts <- rank+1's first zhi_g owned planes
+        stencil_plan_s* Q = c->peers[c->rank + 1];
+        int64_t hq[8];
+        slab_halo(Q->ghost, (int)Q->dims[0], tl * Q->pat.zlo, tl * Q->pat.zhi, c->rank + 1, c->nranks, hq);
+        SM_CUDA(cudaStreamWaitEvent(c->stream, Q->comm->ev_edge, 0));
+        SM_CUDA(cudaMemcpyAsync((char*)bufs[k] + h[6] * pb, (const char*)bufs[k + 1] + hq[2] * pb, h[7] * pb,
+                                cudaMemcpyDeviceToDevice, c->stream));
+      }
+    }
+    SM_CUDA(cudaEventRecord(c->ev_comm, c->stream));
+  }
+  return STENCIL_OK;
+}
+
+// main stream of plan k waits for the exchange that filled its ghosts and,
+// for LOOPBACK, for its neighbours' copies out of its buffer
+static int wait_exchange(const std::vector<stencil_plan_s*>& Ps) {
+  for (stencil_plan_s* P : Ps) {
+    Comm* c = P->comm;
+    SM_CUDA(cudaStreamWaitEvent(P->stream, c->ev_comm, 0));
+    if (c->transport == TR_LOOPBACK) {
+      if (c->rank > 0) SM_CUDA(cudaStreamWaitEvent(P->stream, c->peers[c->rank - 1]->comm->ev_comm, 0));
+      if (c->rank < c->nranks - 1) SM_CUDA(cudaStreamWaitEvent(P->stream, c->peers[c->rank + 1]->comm->ev_comm, 0));
+    }
+  }
+  return STENCIL_OK;
+}
+
+// The time loop (a6) over a group of local plans: one plan on one GPU, one
+// slab per process (NCCL), or all slabs of a LOOPBACK group. With slabs, each
+// launch computes the edge planes first, starts the halo exchange of those
+// planes on the comm stream and computes the interior meanwhile (a7).
+static int run_group(const std::vector<stencil_plan_s*>& Ps, const std::vector<const void*>& ins,
+                     const std::vector<void*>& outs, int steps) {
+  const size_t np = Ps.size();
+  stencil_plan_s* P0 = Ps[0];
+  const bool slab = P0->comm != nullptr;
+  for (size_t k = 0; k < np; ++k) {
+    stencil_plan_s* P = Ps[k];
+    if (!ins[k] || !outs[k]) SM_FAIL(STENCIL_E_INVAL, "null grid pointer");
+    if (ins[k] == outs[k]) SM_FAIL(STENCIL_E_INVAL, "in and out must be distinct buffers");
+    if ((uintptr_t)ins[k] % 16 || (uintptr_t)outs[k] % 16)
+      SM_FAIL(STENCIL_E_INVAL, "grid pointers must be 16-byte aligned");
+    if (P->var.tt != P0->var.tt || P->var.family != P0->var.family)
+      SM_FAIL(STENCIL_E_INVAL, "plans of a group must use the same OC setting");
+  }
   if (steps < 0) SM_FAIL(STENCIL_E_INVAL, "steps must be >= 0");
-  if ((uintptr_t)in % 16 || (uintptr_t)out % 16) SM_FAIL(STENCIL_E_INVAL, "grid pointers must be 16-byte aligned");
   if (steps == 0) {
-    SM_CUDA(cudaMemcpyAsync(out, in, bytes, cudaMemcpyDeviceToDevice, P->stream));
+    for (size_t k = 0; k < np; ++k) {
+      const int elem = Ps[k]->dtype == STENCIL_F64 ? 8 : 4;
+      const size_t bytes = (size_t)Ps[k]->vdims[0] * Ps[k]->vdims[1] * Ps[k]->vdims[2] * elem;
+      SM_CUDA(cudaMemcpyAsync(outs[k], ins[k], bytes, cudaMemcpyDeviceToDevice, Ps[k]->stream));
+    }
     return STENCIL_OK;
   }
-  const int T = P->var.family == FAM_TILED || P->var.family == FAM_STREAM_TB ? P->var.tt : 1;
+  const int T = P0->var.family == FAM_TILED || P0->var.family == FAM_STREAM_TB ? P0->var.tt : 1;
   const int launches = (steps + T - 1) / T;
-  if (launches >= 2 && (!P->ws || P->ws_bytes < bytes))
-    SM_FAIL(STENCIL_E_STATE, "steps=%d needs a workspace of %zu bytes (stencil_plan_set_workspace)", steps, bytes);
-  SM_TRY(ensure_loaded(P));
-  const GridArg g = make_grid(P, P->var.vx);
-  // a4: frame of the input into every buffer the sweep writes (fixed thereafter)
-  SM_TRY(launch_frame_copy(in, out, elem, g, P->stream));
-  if (launches >= 2) SM_TRY(launch_frame_copy(in, P->ws, elem, g, P->stream));
-  const void* src = in;
-  for (int i = 0; i < launches; ++i) {
-    void* dst = ((launches - 1 - i) % 2 == 0) ? out : P->ws;
-    const int tt = std::min(T, steps - i * T);
-    if (tt == T) {
-      SM_TRY(launch_sweep(P, P->var, P->kern, src, dst, g));
-    } else {
-      Variant v;
-      Kernel k;
-      SM_TRY(get_tb_rem_kernel(P, tt, &v, &k));
-      SM_TRY(launch_sweep(P, v, k, src, dst, g));
+  std::vector<GridArg> gs(np);
+  for (size_t k = 0; k < np; ++k) {
+    stencil_plan_s* P = Ps[k];
+    const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+    const size_t bytes = (size_t)P->vdims[0] * P->vdims[1] * P->vdims[2] * elem;
+    if (launches >= 2 && (!P->ws || P->ws_bytes < bytes))
+      SM_FAIL(STENCIL_E_STATE, "steps=%d needs a workspace of %zu bytes (stencil_plan_set_workspace)", steps, bytes);
+    SM_TRY(ensure_loaded(P));
+    gs[k] = make_grid(P, P->var.vx);
+    // a4: frame of the input into every buffer the sweep writes (fixed thereafter)
+    SM_TRY(launch_frame_copy(ins[k], outs[k], elem, gs[k], P->stream));
+    if (launches >= 2) SM_TRY(launch_frame_copy(ins[k], P->ws, elem, gs[k], P->stream));
+  }
+  if (slab) {   // ghosts of the input: neighbours' current owned planes
+    std::vector<void*> b(np);
+    for (size_t k = 0; k < np; ++k) {
+      b[k] = const_cast<void*>(ins[k]);
+      SM_CUDA(cudaEventRecord(Ps[k]->comm->ev_edge, Ps[k]->stream));
     }
-    src = dst;
+    SM_TRY(exchange(Ps, b, std::min(T, steps)));
+    SM_TRY(wait_exchange(Ps));
+  }
+  std::vector<const void*> src(ins);
+  std::vector<void*> dst(np);
+  for (int i = 0; i < launches; ++i) {
+    const int tl = std::min(T, steps - i * T);
+    const bool more = i + 1 < launches;
+    const int tl_next = more ? std::min(T, steps - (i + 1) * T) : 0;
+    for (size_t k = 0; k < np; ++k) dst[k] = ((launches - 1 - i) % 2 == 0) ? outs[k] : Ps[k]->ws;
+    std::vector<Variant> vs(np);
+    std::vector<Kernel> ks(np);
+    for (size_t k = 0; k < np; ++k) {
+      if (tl == T) { vs[k] = Ps[k]->var; ks[k] = Ps[k]->kern; }
+      else SM_TRY(get_tb_rem_kernel(Ps[k], tl, &vs[k], &ks[k]));
+    }
+    if (slab && more) {
+      const int E = tl_next * std::max(P0->pat.zlo, P0->pat.zhi);
+      for (size_t k = 0; k < np; ++k) {   // edge planes first
+        GridArg g = gs[k];
+        const int c0 = g.cz0, c1 = g.cz1;
+        if (c1 - c0 > 2 * E) {
+          g.cz1 = c0 + E;
+          SM_TRY(launch_sweep(Ps[k], vs[k], ks[k], src[k], dst[k], g));
+          g.cz0 = c1 - E; g.cz1 = c1;
+          SM_TRY(launch_sweep(Ps[k], vs[k], ks[k], src[k], dst[k], g));
+        } else {
+          SM_TRY(launch_sweep(Ps[k], vs[k], ks[k], src[k], dst[k], g));
+        }
+        SM_CUDA(cudaEventRecord(Ps[k]->comm->ev_edge, Ps[k]->stream));
+      }
+      SM_TRY(exchange(Ps, dst, tl_next));
+      for (size_t k = 0; k < np; ++k) {   // interior overlaps the exchange
+        GridArg g = gs[k];
+        if (g.cz1 - g.cz0 > 2 * E) {
+          g.cz0 += E; g.cz1 -= E;
+          SM_TRY(launch_sweep(Ps[k], vs[k], ks[k], src[k], dst[k], g));
+        }
+      }
+      SM_TRY(wait_exchange(Ps));
+    } else {
+      for (size_t k = 0; k < np; ++k) SM_TRY(launch_sweep(Ps[k], vs[k], ks[k], src[k], dst[k], gs[k]));
+    }
+    for (size_t k = 0; k < np; ++k) src[k] = dst[k];
   }
   SM_CUDA(cudaGetLastError());
   return STENCIL_OK;
+}
+
+int run_device(stencil_plan_s* P, const void* in, void* out, int steps) {
+  if (P->comm && P->comm->transport == TR_LOOPBACK)
+    SM_FAIL(STENCIL_E_STATE, "a loopback slab runs with its group (stencil_run_group)");
+  return run_group({P}, {in}, {out}, steps);
 }
 
 }  // namespace smart_rt
@@ -604,6 +729,18 @@ int stencil_plan_create(stencil_plan_t* plan, int ndim, const int64_t* dims, int
   // Default tiles shrink until the shared-memory footprint fits (high-order
   // stencils under TB need smaller tiles); user-given fields are kept.
   const bool user_bz = params && params->bz, user_by = params && params->by, user_bx = params && params->bx;
+  if (!user_bx && family_of(oc, P->params.smem) != FAM_NAIVE) {
+    // keep the default halo tile within one TMA box (<= 256 elements per row)
+    const int elem = dtype == STENCIL_F64 ? 8 : 4;
+    for (;;) {
+      Variant v;
+      v.family = family_of(oc, P->params.smem);
+      v.bx = P->params.bx; v.by = P->params.by; v.bz = P->params.bz; v.vx = P->params.vx;
+      v.m = P->params.merge; v.tt = (oc & STENCIL_OC_TB) ? P->params.tb_steps : 1;
+      if (tma_box(v, P->pat, elem).lx <= 256 || P->params.bx <= 8 * P->params.vx) break;
+      P->params.bx /= 2;
+    }
+  }
   for (int attempt = 0;; ++attempt) {
     const int rc = resolve_variant(P.get());
     if (rc != STENCIL_E_OC_INFEASIBLE || attempt > 12) {
@@ -672,9 +809,8 @@ int stencil_plan_info(stencil_plan_t P, stencil_plan_info_t* info) {
   info->threads = P->var.threads();
   info->regs = P->kern.regs;
   info->uses_tma = P->var.tma ? 1 : 0;
-  long long pts = 1;
-  for (int k = 0; k < 3; ++k) pts *= (P->vdims[k] - 2 * P->frame[k]);
-  info->points = pts;
+  const GridArg g = make_grid(P, P->var.vx);   // points this plan updates per time step
+  info->points = (long long)(g.cz1 - g.cz0) * (g.cy1 - g.cy0) * (g.cx1 - g.cx0);
   snprintf(info->kernel_name, sizeof info->kernel_name, "%s", P->lowered.c_str());
   return STENCIL_OK;
 }
@@ -701,6 +837,22 @@ int stencil_plan_kernel_time(stencil_plan_t P, double* kernel_ms, int64_t* launc
   *launches = (int64_t)(P->ev_used / 2);
   P->ev_used = 0;
   return STENCIL_OK;
+}
+
+int stencil_run_group(stencil_plan_t* plans, int nplans, const void* const* ins, void* const* outs, int steps) {
+  clear_error();
+  if (!plans || !ins || !outs || nplans < 1) SM_FAIL(STENCIL_E_INVAL, "bad arguments");
+  std::vector<stencil_plan_s*> ps(plans, plans + nplans);
+  for (int k = 0; k < nplans; ++k) {
+    if (!ps[k]) SM_FAIL(STENCIL_E_INVAL, "null plan %d", k);
+    Comm* c = ps[k]->comm;
+    if (nplans > 1 && (!c || c->transport != TR_LOOPBACK || c->nranks != nplans || c->rank != k ||
+                       c->peers[k] != ps[k]))
+      SM_FAIL(STENCIL_E_STATE, "plans must be one loopback group in rank order");
+  }
+  if (nplans == 1 && ps[0]->comm && ps[0]->comm->transport == TR_LOOPBACK && ps[0]->comm->nranks != 1)
+    SM_FAIL(STENCIL_E_STATE, "a loopback slab runs with its whole group");
+  return run_group(ps, std::vector<const void*>(ins, ins + nplans), std::vector<void*>(outs, outs + nplans), steps);
 }
 
 int stencil_run(stencil_plan_t plan, const void* in, void* out, int steps) {

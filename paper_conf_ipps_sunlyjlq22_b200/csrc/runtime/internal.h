@@ -115,8 +115,30 @@ int launch_fill(void* dst, int dtype, const int64_t box[3], const int64_t org[3]
                 uint64_t seed, int kind, cudaStream_t s);
 
 // ---------------------------------------------------------------- comm
-struct Comm;
+// Slab decomposition along the slowest axis. A plan with a
+// communicator owns `n = dims[0]` planes stored after G ghost planes, followed
+// by G more: the device array has n + 2G planes. Transport: NCCL send/recv
+// between processes, or LOOPBACK (all slabs as plans of one process, halos by
+// cudaMemcpyAsync -- the multi-GPU schedule exercised on one device).
+enum Transport { TR_NONE = 0, TR_NCCL = 1, TR_LOOPBACK = 2 };
+
+struct Comm {
+  int transport = TR_NONE;
+  int rank = 0, nranks = 1;
+  bool owner = true;                 // owns the NCCL communicator
+  void* nccl = nullptr;              // ncclComm_t
+  cudaStream_t stream = nullptr;     // comm stream (owned per plan)
+  cudaEvent_t ev_edge = nullptr;     // edge planes of dst written (main stream)
+  cudaEvent_t ev_comm = nullptr;     // halo exchange into dst done (comm stream)
+  std::vector<stencil_plan_s*> peers;  // LOOPBACK: plans of all ranks (index = rank)
+  const void* cur = nullptr;         // LOOPBACK: buffer this rank is exchanging (for peers)
+};
 void comm_destroy(Comm* c);
+int comm_create_stream_events(Comm* c);
+// Halo plane ranges (local plane indices) of a launch fusing `tl` steps.
+void slab_halo(int ghost, int n, int zlo_g, int zhi_g, int rank, int nranks, int64_t out[8]);
+int comm_exchange_nccl(stencil_plan_s* P, void* buf, int tl);
+int comm_allreduce_max(stencil_plan_s* P, float* v, int n);
 
 // ---------------------------------------------------------------- plan
 struct stencil_plan_impl;
@@ -136,8 +158,9 @@ struct stencil_plan_s {
 
   // kernel view (3-D)
   smart_rt::Pattern pat;
-  int64_t vdims[3] = {0, 0, 0};  // view extents nz, ny, nx
+  int64_t vdims[3] = {0, 0, 0};  // view extents nz, ny, nx (with ghosts: n + 2G planes)
   int frame[3] = {0, 0, 0};      // frame widths per view axis
+  int ghost = 0;                 // G: ghost planes on each side of the slab (0 = no slab)
   smart_rt::Variant var;
   std::string src;               // generated source of the main variant
   std::string lowered;
