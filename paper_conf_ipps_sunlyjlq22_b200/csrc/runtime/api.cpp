@@ -246,7 +246,8 @@ static int resolve_variant(stencil_plan_s* P) {
   const int fam = family_of(P->oc, p.smem);
   Variant v;
   v.family = fam;
-  v.bx = p.bx; v.by = p.by; v.bz = p.bz; v.vx = p.vx; v.m = p.merge;
+  v.bx = p.bx; v.by = p.by; v.bz = p.bz; v.vx = p.vx;
+  v.m = (P->oc & (STENCIL_OC_BM | STENCIL_OC_CM)) ? p.merge : 1;   // merging only under BM / CM
   v.cm = (P->oc & STENCIL_OC_CM) != 0;
   v.tt = (P->oc & STENCIL_OC_TB) ? p.tb_steps : 1;
   v.rt = (P->oc & STENCIL_OC_RT) != 0;
@@ -724,6 +725,10 @@ int stencil_plan_create(stencil_plan_t* plan, int ndim, const int64_t* dims, int
   P->coeffs.assign(coeffs, coeffs + tsize);
   default_params(oc, ndim, dtype, &P->params);
   merge_params(params, &P->params);
+  // parameters an OC does not have are reported at their neutral value
+  if (!(oc & (STENCIL_OC_BM | STENCIL_OC_CM))) P->params.merge = 1;
+  if (!(oc & STENCIL_OC_TB)) P->params.tb_steps = 1;
+  if (!(oc & STENCIL_OC_PR)) P->params.pr_stages = 1;
   SM_TRY(build_pattern(P.get()));
   build_view(P.get(), family_of(oc, P->params.smem));
   // Default tiles shrink until the shared-memory footprint fits (high-order
