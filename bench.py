@@ -249,17 +249,21 @@ def run_impl(args):
     peak, peak_kind = _peaks()
 
     slab = (world > 1 or args.slab) and len(dims) == 3
-    uid = None
-    if slab:   # NCCL unique id for the library's own communicator (a7)
-        obj = [sm.nccl_unique_id() if rank == 0 else None]
-        if world > 1:
-            dist.broadcast_object_list(obj, src=0)
-        uid = obj[0]
+    comm_owner = []
 
     def make_plan(oc, params=None):
+        """Plan on this rank's slab; the halo exchange (a7) runs on torch's NCCL
+        communicator (N > 1) or on one library-owned communicator (N = 1)."""
         p = sm.Plan(dims, acc, c, dtype, oc, params)
         if slab:
-            p.set_comm(uid, rank, world)
+            if world > 1:
+                be = dist.distributed_c10d._get_default_group()._get_backend(dev)
+                p.set_nccl_comm(be._comm_ptr(), rank, world)
+            elif comm_owner:
+                p.share_comm(comm_owner[0])
+            else:
+                p.set_comm(sm.nccl_unique_id(), rank, world)
+                comm_owner.append(p)
         return p
 
     # every rank owns dims[0] planes of a global grid of depth world*dims[0]
@@ -352,18 +356,34 @@ def run_impl(args):
     value = pts_all * steps / (ms_per_step * 1e-3) / 1e9
 
     # ---- 3. roofline of the dominant kernel (the labelled OC's sweep kernel)
+    # A "launch" here is one application of the kernel to the whole owned grid
+    # (with slabs it is split into edge + interior pieces; their times add up).
     T = pinfo["params"]["tb_steps"] if best_oc & sm.OC_TB else 1
+    groups = args.steps * math.ceil(steps / T)
     bytes_per_launch = pts * 2 * elem          # read + write each interior point once per launch
-    avg_launch_ms = kern_ms / max(kern_n, 1)
+    flops_per_step = pts * 2 * pinfo["nnz"]    # one FMA per neighbour per point and step
+    avg_launch_ms = kern_ms / max(groups, 1)
     achieved = bytes_per_launch / (avg_launch_ms * 1e-3) / 1e9
+    # FP64 148 SM x 64 FMA/clk x 2 x 1.965 GHz = 37.2 TFLOP/s; FP32 x2
+    fp_peak = 148 * 64 * 2 * 1.965e9 / 1e12 * (1 if dtype == "f64" else 2)
+    achieved_fp = flops_per_step * args.steps * steps / (kern_ms * 1e-3) / 1e12
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4),
                 "traffic": _traffic_from_profiles(kernel_key(name, pinfo["kernel_name"])),
                 "peak_kind": peak_kind, "kernel": kernel_key(name, pinfo["kernel_name"]),
-                "launch_ms": round(avg_launch_ms, 4),
+                "launch_ms": round(avg_launch_ms, 4), "launches": kern_n,
                 "kernel_share_of_step": round(kern_ms / max(total_ms, 1e-9), 4),
                 "bytes_per_launch": bytes_per_launch, "time_steps_per_launch": T,
-                "frac_of_spec_8tbs": round(achieved / HBM_SPEC_GBS, 4)}
+                "frac_of_spec_8tbs": round(achieved / HBM_SPEC_GBS, 4),
+                "fp": {"achieved": round(achieved_fp, 2), "peak": round(fp_peak, 1), "unit": "TFLOP/s",
+                       "frac": round(achieved_fp / fp_peak, 4), "peak_kind": "derived (DESIGN.md §6)"}}
+    if achieved_fp / fp_peak > achieved / peak:   # FMA-bound stencil (C4, high-order random)
+        roofline.update({"bound": "alu", "achieved": round(achieved_fp, 2), "peak": round(fp_peak, 1),
+                         "unit": "TFLOP/s", "frac": round(achieved_fp / fp_peak, 4),
+                         "peak_kind": "derived (DESIGN.md §6)",
+                         "hbm": {"achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                                 "frac": round(achieved / peak, 4)}})
+        roofline.pop("fp")
 
     # ---- 4. e2e through the public API with host buffers
     e2e = None

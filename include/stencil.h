@@ -239,6 +239,16 @@ int stencil_nccl_unique_id(uint8_t *id);
  * owned planes. Collective: all ranks call it with the same id; tb_steps <= 4. */
 int stencil_plan_set_comm(stencil_plan_t plan, const uint8_t *id, int rank, int nranks);
 
+/* Same as stencil_plan_set_comm, but adopting an existing NCCL communicator
+ * (an ncclComm_t, e.g. the one torch.distributed's NCCL process group owns);
+ * the plan does not destroy it. The communicator must span `nranks` ranks with
+ * this process at `rank`, on the current device, and outlive the plan. */
+int stencil_plan_set_nccl_comm(stencil_plan_t plan, void *nccl_comm, int rank, int nranks);
+
+/* Attach `plan` to the communicator of `src` (set by either call above; a
+ * unique id initialises only one communicator). `src` must outlive `plan`. */
+int stencil_plan_share_comm(stencil_plan_t plan, stencil_plan_t src);
+
 /* Single-device test form of the decomposition: link `nranks` plans of one
  * process (rank k = plans[k], same stencil/OC/dtype/plane shape) as slabs of one
  * global grid; halos move by cudaMemcpyAsync between their buffers, with the

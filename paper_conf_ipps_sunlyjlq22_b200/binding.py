@@ -93,6 +93,8 @@ _SIGS = {
     "stencil_slab_range": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int, ctypes.c_int,
                                           ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64)]),
     "stencil_plans_link_loopback": (ctypes.c_int, [ctypes.POINTER(ctypes.c_void_p), ctypes.c_int]),
+    "stencil_plan_set_nccl_comm": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int, ctypes.c_int]),
+    "stencil_plan_share_comm": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "stencil_run_group": (ctypes.c_int, [ctypes.POINTER(ctypes.c_void_p), ctypes.c_int,
                                          ctypes.POINTER(ctypes.c_void_p), ctypes.POINTER(ctypes.c_void_p),
                                          ctypes.c_int]),
@@ -380,8 +382,17 @@ class Plan:
         return float(ms.value), int(n.value)
 
     def set_comm(self, uid: bytes, rank: int, nranks: int) -> None:
+        """New NCCL communicator from a unique id (one communicator per id)."""
         buf = (ctypes.c_uint8 * 128).from_buffer_copy(uid)
         _check(lib().stencil_plan_set_comm(self._h, buf, rank, nranks))
+
+    def set_nccl_comm(self, comm_ptr: int, rank: int, nranks: int) -> None:
+        """Adopt an existing ncclComm_t (e.g. torch's: ProcessGroupNCCL._comm_ptr())."""
+        _check(lib().stencil_plan_set_nccl_comm(self._h, ctypes.c_void_p(comm_ptr), rank, nranks))
+
+    def share_comm(self, other: "Plan") -> None:
+        self._comm_src = other          # keep the owner alive
+        _check(lib().stencil_plan_share_comm(self._h, other._h))
 
 
 def gstencil_per_s(points: int, steps: int, ms: float) -> float:

@@ -155,6 +155,27 @@ extern "C" int stencil_plan_set_comm(stencil_plan_t P, const uint8_t* id, int ra
   return STENCIL_OK;
 }
 
+extern "C" int stencil_plan_set_nccl_comm(stencil_plan_t P, void* nccl_comm, int rank, int nranks) {
+  clear_error();
+  if (!P || !nccl_comm) SM_FAIL(STENCIL_E_INVAL, "null argument");
+  if (nranks < 1 || rank < 0 || rank >= nranks) SM_FAIL(STENCIL_E_INVAL, "bad rank/nranks");
+  int n = 0, r = 0;
+  if (ncclCommCount((ncclComm_t)nccl_comm, &n) != ncclSuccess || ncclCommUserRank((ncclComm_t)nccl_comm, &r) != ncclSuccess ||
+      n != nranks || r != rank)
+    SM_FAIL(STENCIL_E_INVAL, "communicator does not match rank %d of %d", rank, nranks);
+  SM_TRY(slab_setup(P, rank, nranks, TR_NCCL));
+  P->comm->nccl = nccl_comm;
+  P->comm->owner = false;
+  return STENCIL_OK;
+}
+
+extern "C" int stencil_plan_share_comm(stencil_plan_t P, stencil_plan_t src) {
+  clear_error();
+  if (!P || !src || !src->comm || src->comm->transport != TR_NCCL)
+    SM_FAIL(STENCIL_E_INVAL, "source plan has no NCCL communicator");
+  return stencil_plan_set_nccl_comm(P, src->comm->nccl, src->comm->rank, src->comm->nranks);
+}
+
 extern "C" int stencil_plans_link_loopback(stencil_plan_t* plans, int nranks) {
   clear_error();
   if (!plans || nranks < 1) SM_FAIL(STENCIL_E_INVAL, "bad arguments");
