@@ -208,6 +208,42 @@ int stencil_sample_params(uint32_t oc, int ndim, stencil_dtype_t dtype, uint64_t
                           stencil_params_t *out);
 
 /* ---------------------------------------------------------------------------
+ * Stencil representation (§IV-C; host only)
+ * ------------------------------------------------------------------------- */
+
+/* Table II feature set: order = maximum (Chebyshev) extent of the
+ * non-zeros, nnz, sparsity = nnz / 9^ndim (the fixed (2*4+1)^d tensor of
+ * P:L135), nnz_order[n-1] = non-zeros in ring n, nnz_ratio[n-1] =
+ * nnz_order[n-1] / |ring n| (|ring n| = (2n+1)^d - (2n-1)^d). */
+typedef struct {
+    int32_t order;
+    int32_t nnz;
+    double sparsity;
+    int32_t nnz_order[4];
+    double nnz_ratio[4];
+} stencil_features_t;
+
+int stencil_features(int ndim, int order, const uint8_t *access, stencil_features_t *out);
+
+/* The access tensor embedded, centred, in the fixed 9^ndim binary tensor of
+ * Fig. 6 (the ConvNet / ConvMLP input). out9: 729 (3-D) or 81 bytes. */
+int stencil_embed_tensor(int ndim, int order, const uint8_t *access, uint8_t *out9);
+
+/* Rows of the last stencil_oc_sweep on `plan` (the paper's stencil dataset:
+ * "each parameter setting and its corresponding execution time are also
+ * stored"): one row per (OC, setting) tried, in sweep order. Writes at
+ * most max_rows rows and the total count to *nrows. time_ms = +INF if the
+ * setting was infeasible. */
+typedef struct {
+    uint32_t oc;
+    int32_t setting;          /* k of stencil_sample_params */
+    stencil_params_t params;  /* resolved setting (defaults filled in) */
+    float time_ms;            /* median of the timed runs */
+} stencil_sweep_row_t;
+
+int stencil_sweep_rows(stencil_plan_t plan, stencil_sweep_row_t *rows, int max_rows, int *nrows);
+
+/* ---------------------------------------------------------------------------
  * Synthetic inputs (the counter-based generator of DESIGN.md, reading C-3)
  * ------------------------------------------------------------------------- */
 

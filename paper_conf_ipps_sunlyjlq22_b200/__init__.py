@@ -5,10 +5,12 @@ combination (OC) of Table I, and the per-OC timing sweep that labels the best
 OC. Compute lives in libstencilmart.so (C ABI: include/stencil.h); this package
 is its thin ctypes binding.
 """
-from .binding import (F32, F64, NUM_OC, OC_BM, OC_CM, OC_PR, OC_RT, OC_ST, OC_TB, Plan, StencilError, link_loopback, run_group, slab_halo,
-                      exported_symbols, fill_field, gstencil_per_s, launch_count, lib, nccl_unique_id,
-                      oc_from_name, oc_list, oc_name, oc_valid, sample_params, slab_range)
+from .binding import (F32, F64, NUM_OC, OC_BM, OC_CM, OC_PR, OC_RT, OC_ST, OC_TB, Plan, StencilError,
+                      embed_tensor, exported_symbols, features, fill_field, gstencil_per_s, launch_count, lib,
+                      link_loopback, nccl_unique_id, oc_from_name, oc_list, oc_name, oc_valid, run_group,
+                      sample_params, slab_halo, slab_range)
 
-__all__ = ["link_loopback", "run_group", "slab_halo", "F32", "F64", "NUM_OC", "OC_BM", "OC_CM", "OC_PR", "OC_RT", "OC_ST", "OC_TB", "Plan",
-           "StencilError", "exported_symbols", "fill_field", "gstencil_per_s", "launch_count", "lib",
-           "nccl_unique_id", "oc_from_name", "oc_list", "oc_name", "oc_valid", "sample_params", "slab_range"]
+__all__ = ["F32", "F64", "NUM_OC", "OC_BM", "OC_CM", "OC_PR", "OC_RT", "OC_ST", "OC_TB", "Plan", "StencilError",
+           "embed_tensor", "exported_symbols", "features", "fill_field", "gstencil_per_s", "launch_count", "lib",
+           "link_loopback", "nccl_unique_id", "oc_from_name", "oc_list", "oc_name", "oc_valid", "run_group",
+           "sample_params", "slab_halo", "slab_range"]

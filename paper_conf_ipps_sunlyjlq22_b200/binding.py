@@ -61,9 +61,23 @@ class PlanInfo(ctypes.Structure):
                 ("points", ctypes.c_int64), ("kernel_name", ctypes.c_char * 128)]
 
 
+class Features(ctypes.Structure):
+    _fields_ = [("order", ctypes.c_int32), ("nnz", ctypes.c_int32), ("sparsity", ctypes.c_double),
+                ("nnz_order", ctypes.c_int32 * 4), ("nnz_ratio", ctypes.c_double * 4)]
+
+
+class SweepRow(ctypes.Structure):
+    _fields_ = [("oc", ctypes.c_uint32), ("setting", ctypes.c_int32), ("params", Params),
+                ("time_ms", ctypes.c_float)]
+
+
 _lib = None
 
 _SIGS = {
+    "stencil_features": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.POINTER(Features)]),
+    "stencil_embed_tensor": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p]),
+    "stencil_sweep_rows": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(SweepRow), ctypes.c_int,
+                                          ctypes.POINTER(ctypes.c_int)]),
     "stencil_plan_create": (ctypes.c_int, [ctypes.POINTER(ctypes.c_void_p), ctypes.c_int,
                                            ctypes.POINTER(ctypes.c_int64), ctypes.c_int, ctypes.c_void_p,
                                            ctypes.c_void_p, ctypes.c_int, ctypes.c_uint32,
@@ -186,6 +200,27 @@ def slab_range(nz_global: int, rank: int, nranks: int) -> Tuple[int, int]:
     a, b = ctypes.c_int64(), ctypes.c_int64()
     _check(lib().stencil_slab_range(nz_global, rank, nranks, ctypes.byref(a), ctypes.byref(b)))
     return int(a.value), int(b.value)
+
+
+def features(access: np.ndarray) -> Dict[str, float]:
+    """Table II features of an access tensor, same keys as oracle.features."""
+    acc = np.ascontiguousarray(access, dtype=np.uint8)
+    order = (acc.shape[0] - 1) // 2
+    f = Features()
+    _check(lib().stencil_features(acc.ndim, order, acc.ctypes.data, ctypes.byref(f)))
+    out: Dict[str, float] = {"order": f.order, "nnz": f.nnz, "sparsity": f.sparsity}
+    for n in range(4):
+        out[f"nnz_order{n + 1}"] = f.nnz_order[n]
+        out[f"nnzRatio_order{n + 1}"] = f.nnz_ratio[n]
+    return out
+
+
+def embed_tensor(access: np.ndarray) -> np.ndarray:
+    """The access tensor centred in the fixed 9^d tensor of Fig. 6."""
+    acc = np.ascontiguousarray(access, dtype=np.uint8)
+    out = np.zeros((9,) * acc.ndim, dtype=np.uint8)
+    _check(lib().stencil_embed_tensor(acc.ndim, (acc.shape[0] - 1) // 2, acc.ctypes.data, out.ctypes.data))
+    return out
 
 
 def slab_halo(ghost: int, n: int, zlo_g: int, zhi_g: int, rank: int, nranks: int) -> Dict[str, Tuple[int, int]]:
@@ -365,11 +400,17 @@ class Plan:
         _check(L.stencil_oc_sweep(self._h, ctypes.c_void_p(inp.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                                   int(steps), int(settings_per_oc), int(reps), int(seed), times, ids, bp,
                                   ctypes.byref(best)))
+        n = ctypes.c_int()
+        _check(L.stencil_sweep_rows(self._h, None, 0, ctypes.byref(n)))
+        rows = (SweepRow * max(n.value, 1))()
+        _check(L.stencil_sweep_rows(self._h, rows, n.value, ctypes.byref(n)))
         return {
             "times_ms": [float(times[i]) for i in range(NUM_OC)],
             "oc_ids": [int(ids[i]) for i in range(NUM_OC)],
             "best_params": [bp[i].to_dict() for i in range(NUM_OC)],
             "best_oc": int(best.value),
+            "rows": [{"oc": int(r.oc), "oc_name": oc_name(r.oc), "setting": int(r.setting),
+                      "params": r.params.to_dict(), "time_ms": float(r.time_ms)} for r in rows[:n.value]],
         }
 
     def set_timing(self, enable: bool) -> None:

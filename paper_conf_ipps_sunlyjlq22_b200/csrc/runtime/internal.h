@@ -181,6 +181,9 @@ struct stencil_plan_s {
   void* h_out_dev = nullptr;
   void* h_ws_dev = nullptr;
 
+  // rows of the last OC sweep (stencil_sweep_rows)
+  std::vector<stencil_sweep_row_t> sweep_rows;
+
   // kernel timing (stencil_plan_set_timing)
   bool timing = false;
   std::vector<cudaEvent_t> ev_pool;      // pairs: [2i] before, [2i+1] after launch i

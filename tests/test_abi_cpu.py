@@ -141,3 +141,23 @@ def test_2d_plans():
     for oc in (0, sm.OC_ST, sm.OC_TB, sm.OC_BM):
         p = _plan((256, 256), acc, c, "f64", oc)
         assert p.info["ndim"] == 2 and p.info["points"] == 254 * 254
+
+
+@pytest.mark.parametrize("ndim", [2, 3])
+def test_table2_features_match_oracle(ndim):
+    """Table II extractor in the C ABI == the oracle's statement, bit for bit."""
+    for order in (1, 2, 3, 4):
+        for seed in range(3):
+            acc, _ = si.random_stencil(ndim, order, seed)
+            assert sm.features(acc) == oracle.features(acc)
+        for acc in (si.star(ndim, order, 1.0, [1.0] * order)[0], si.box(ndim, order, 1.0, 1.0)[0]):
+            assert sm.features(acc) == oracle.features(acc)
+
+
+def test_embed_tensor_centred():
+    acc, _ = si.random_stencil(3, 2, 4)
+    t9 = sm.embed_tensor(acc)
+    assert t9.shape == (9, 9, 9) and t9.sum() == acc.sum() and t9[4, 4, 4] == 1
+    assert np.array_equal(t9[2:7, 2:7, 2:7], acc)
+    acc2, _ = si.random_stencil(2, 4, 1)
+    assert np.array_equal(sm.embed_tensor(acc2), acc2)
