@@ -89,8 +89,8 @@ typedef struct {
     int32_t merge;        /* BM/CM merge factor k (outputs per thread along y; 1..8) */
     int32_t stream_chunk; /* ST: output planes per CTA ("concurrent streaming") */
     int32_t tb_steps;     /* TB: time steps fused per launch (2..8) */
-    int32_t pr_stages;    /* PR: planes in flight in the TMA pipeline (enumeration 1..4;
-                             1 = no prefetching) */
+    int32_t pr_stages;    /* PR: planes in flight in the TMA pipeline (1..8; the settings
+                             sampler draws the enumeration 2..4; 1 = no prefetching) */
     int32_t reserved[3];  /* must be 0 */
 } stencil_params_t;
 

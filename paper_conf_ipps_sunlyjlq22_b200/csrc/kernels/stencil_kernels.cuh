@@ -59,6 +59,19 @@ __device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;"
                :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
 }
+__device__ __forceinline__ void mbar_arrive(unsigned long long* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
+}
+// wait with a suspend-time hint: the warp sleeps in the barrier unit instead of
+// spinning through issue slots (warp-specialised pipelines wait a lot)
+__device__ __forceinline__ void mbar_wait_sleep(unsigned long long* bar, unsigned parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, %2;\n\t"
+      "@!P1 bra WAIT_%=;\n\t}"
+      :: "r"(smem_u32(bar)), "r"(parity), "r"(0x989680u) : "memory");
+}
 __device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned parity) {
   asm volatile(
       "{\n\t.reg .pred P1;\n"
@@ -226,14 +239,14 @@ __device__ __forceinline__ void run_gather(const L (&pl)[S::NZ], typename S::T (
   run_gather_ops<S, S, VX, M>(pl, acc);
 }
 
-template <class S, int VX, int M, int U, class L>
-__device__ __forceinline__ void run_scatter(const L& pl, typename S::T (&acc)[S::NZ][M][VX]) {
+template <class S, class O, int VX, int M, int U, class L>
+__device__ __forceinline__ void run_scatter_ops(const L& pl, typename S::T (&acc)[S::NZ][M][VX]) {
   typedef typename S::T T;
   constexpr int NZ = S::NZ;
   T w[VX];
 #pragma unroll
-  for (int i = 0; i < S::NOPS; ++i) {
-    const unsigned op = S::op(i);
+  for (int i = 0; i < O::NOPS; ++i) {
+    const unsigned op = O::op(i);
     if (!(op >> 31)) {
       pl.get(int((op >> 4) & 255) - 128, int((op >> 12) & 15) - 8, w);
     } else {
@@ -242,6 +255,11 @@ __device__ __forceinline__ void run_scatter(const L& pl, typename S::T (&acc)[S:
       a = fma_t(S::coef(op & 1023), w[(op >> 10) & 3], a);
     }
   }
+}
+
+template <class S, int VX, int M, int U, class L>
+__device__ __forceinline__ void run_scatter(const L& pl, typename S::T (&acc)[S::NZ][M][VX]) {
+  run_scatter_ops<S, S, VX, M, U>(pl, acc);
 }
 
 // Store a thread tile (rows given by the merge mode) into global memory,
@@ -772,6 +790,267 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
         store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc);
       }
       __syncthreads();
+    }
+  }
+}
+
+// ===========================================================================
+// Streaming + temporal blocking with retiming in EVERY fused step: the OCs
+// ST_TB_RT and their BM/CM/PR combinations.
+// Retiming (split partial sums) lets each stage consume only the NEWEST plane
+// of the stage below it: stage s keeps, per thread tile, a register queue of
+// NZ partial-sum planes; when input plane q of stage s-1 arrives, every value
+// of its window is scattered into the NZ live outputs, and output plane
+// q - ZHI completes and is written to stage s's shared-memory plane. A stage
+// therefore reads ONE plane window from shared memory per output tile (the
+// gather pipeline k_stream_tb reads NZ), so shared-memory traffic per fused
+// step is about that of one ST sweep while HBM traffic is divided by TT.
+//
+// Warp-specialised pipeline (no CTA-wide barrier in the loop):
+//   warp 0, lane 0  producer: TMA loads of input planes into an NS-slot ring
+//                   (NS = planes in flight: PR; NS = 1 is "no prefetching");
+//   group s=1..TT-1 one VX x MI register tile per thread over region R_s
+//                   (the output tile expanded by (TT-s)*extent), op table
+//                   S::Mid in scatter form; writes stage-s planes into a
+//                   2-slot ring;
+//   group TT        the M x VX (BM/CM) output tile of k_stream, scatter form,
+//                   stores to HBM.
+// Hand-offs are mbarriers: full[slot] (count = producer threads; TMA: tx
+// bytes) and empty[slot] (count = consumer threads), parity = use count & 1.
+// Groups run decoupled; a group waits only when its input is not ready or
+// its output slot is still being read.
+//
+// Tile values outside R_s are computed from don't-care inputs and never feed
+// a valid output, so they are stored unmasked (inside the plane buffer).
+// Frame points (outside the update box) keep their value at every fused step
+// and read it from the launch's input grid (the frame never changes,
+// DESIGN.md C-1). Canonical order (C-4): partial sums receive slices in
+// ascending dz and, in each slice, FMAs in (dy,dx) order -- bitwise equal to
+// every other OC.
+// ===========================================================================
+template <class S, int BX, int BY, int VX, int M, int TT, int MI, int s>
+struct TbRtStage {
+  static constexpr int HX0 = (TT - s) * S::XLO, HX1 = (TT - s) * S::XHI;
+  static constexpr int HY0 = (TT - s) * S::YLO, HY1 = (TT - s) * S::YHI;
+  static constexpr int TXL = ((HX0 + VX - 1) / VX) * VX;   // tile x origin = xb - TXL
+  static constexpr int NTX = (TXL + BX + HX1 + VX - 1) / VX;
+  static constexpr int RY = BY * M + HY0 + HY1;
+  static constexpr int NTY = (RY + MI - 1) / MI;
+  static constexpr int NT = NTX * NTY;
+  static constexpr int W = (NT + 31) / 32;                 // warps of group s
+};
+
+// first warp of group s (1..TT; group TT = the last stage); warp 0 = producer
+template <class S, int BX, int BY, int VX, int M, int TT, int MI, int s>
+struct TbRtWarp0 {
+  static constexpr int value =
+      TbRtWarp0<S, BX, BY, VX, M, TT, MI, s - 1>::value + TbRtStage<S, BX, BY, VX, M, TT, MI, s - 1>::W;
+};
+template <class S, int BX, int BY, int VX, int M, int TT, int MI>
+struct TbRtWarp0<S, BX, BY, VX, M, TT, MI, 1> { static constexpr int value = 1; };
+
+template <class S, int BX, int BY, int VX, int M, bool CM, int NS, int TT>
+struct StreamTbRtCfg {
+  typedef typename S::T T;
+  static constexpr int ALN = (16 / (int)sizeof(T)) > VX ? (16 / (int)sizeof(T)) : VX;
+  static constexpr int XOFF = ((TT * S::XLO + ALN - 1) / ALN) * ALN;
+  static constexpr int LX = ((XOFF + BX + TT * S::XHI + ALN - 1) / ALN) * ALN;
+  static constexpr int LY = BY * M + TT * (S::YLO + S::YHI);
+  static constexpr int PLANE = ((LX * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
+  static constexpr int MI = S::MI;
+  static constexpr int PADF = 128 / (int)sizeof(T);
+  static constexpr int PADB = ((MI * LX + ALN) * (int)sizeof(T) + 127) / 128 * 128 / (int)sizeof(T);
+  static constexpr int ELEMS = PADF + (NS + 2 * (TT - 1)) * PLANE + PADB;
+  static constexpr int NBAR = 2 * NS + 4 * (TT - 1);
+  static constexpr int SMEM = ELEMS * (int)sizeof(T) + 8 * NBAR + 128;
+  static constexpr int FT = (BX / VX) * BY;                 // last-stage tiles
+  static constexpr int WF = (FT + 31) / 32;
+  static constexpr int WL = TbRtWarp0<S, BX, BY, VX, M, TT, MI, TT>::value;   // first last-stage warp
+  static constexpr int THREADS = 32 * (WL + WF);
+};
+
+template <class S, int BX, int BY, int VX, int M, bool CM, int NS, int TT>
+__global__ void __launch_bounds__(StreamTbRtCfg<S, BX, BY, VX, M, CM, NS, TT>::THREADS, S::MINB)
+k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, Grid g, int chunk,
+               const __grid_constant__ TmaDesc tmap) {
+  typedef typename S::T T;
+  typedef StreamTbRtCfg<S, BX, BY, VX, M, CM, NS, TT> C;
+  constexpr int NZ = S::NZ;
+  constexpr int MI = C::MI;
+  static_assert(TT >= 2, "k_stream_tb_rt needs TT >= 2");
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  T* sbase = reinterpret_cast<T*>(smem_raw);
+  T* ring0 = sbase + C::PADF;
+  T* mid = ring0 + NS * C::PLANE;                      // stage s slot b: mid + (2*(s-1)+b)*PLANE
+  unsigned long long* bars = reinterpret_cast<unsigned long long*>(smem_raw + C::ELEMS * sizeof(T));
+  // bars: full_in[NS], empty_in[NS], then per stage s=1..TT-1: full_s[2], empty_s[2]
+  unsigned long long* full_in = bars;
+  unsigned long long* empty_in = bars + NS;
+  auto full_s = [&](int s) { return bars + 2 * NS + 4 * (s - 1); };
+  auto empty_s = [&](int s) { return bars + 2 * NS + 4 * (s - 1) + 2; };
+
+  const int tid = threadIdx.x;
+  const int warp = tid >> 5;
+  const int xa = (g.cx0 / C::ALN) * C::ALN;
+  const int xb = xa + blockIdx.x * BX;
+  const int yb = g.cy0 + blockIdx.y * BY * M;
+  const int zs = g.cz0 + blockIdx.z * chunk;
+  const int ze = min(zs + chunk, g.cz1);
+  const int pin0 = zs - TT * S::ZLO;                   // first input plane
+  const int nin = (ze - zs) + TT * (NZ - 1);           // planes each stage consumes
+  const int X0 = xb - C::XOFF, Y0 = yb - TT * S::YLO;
+
+  // stage planes start defined (their unwritten corners only feed discarded outputs)
+  for (int i = tid; i < C::ELEMS; i += C::THREADS) sbase[i] = T(0);
+  if (tid == 0) {
+    tma_prefetch_desc(&tmap);
+    for (int q = 0; q < NS; ++q) {
+      mbar_init(&full_in[q], 1);
+      mbar_init(&empty_in[q], 32 * TbRtStage<S, BX, BY, VX, M, TT, MI, 1>::W);
+    }
+    static_for<1, TT>([&](auto sc) {
+      constexpr int s = decltype(sc)::value;
+      constexpr int WN = s + 1 < TT ? TbRtStage<S, BX, BY, VX, M, TT, MI, s + 1>::W : C::WF;
+      for (int b = 0; b < 2; ++b) {
+        mbar_init(&full_s(s)[b], 32 * TbRtStage<S, BX, BY, VX, M, TT, MI, s>::W);
+        mbar_init(&empty_s(s)[b], 32 * WN);
+      }
+    });
+    fence_mbar_init();
+  }
+  fence_proxy_async();                                  // generic zero-fill before async-proxy writes
+  __syncthreads();
+
+  // ------------------------------------------------------------ producer
+  if (warp == 0) {
+    if (tid == 0) {
+#pragma unroll 1
+      for (int j = 0; j < nin; ++j) {
+        const int slot = j % NS;
+        if (j >= NS) mbar_wait_sleep(&empty_in[slot], (unsigned)((j / NS - 1) & 1));
+        mbar_expect_tx(&full_in[slot], C::LX * C::LY * (unsigned)sizeof(T));
+        tma_load_3d(ring0 + slot * C::PLANE, &tmap, &full_in[slot], X0, Y0, pin0 + j);
+      }
+    }
+    return;
+  }
+
+  // ------------------------------------------------------------ intermediate stages
+  bool done = false;
+  static_for<1, TT>([&](auto sc) {
+    constexpr int s = decltype(sc)::value;
+    typedef TbRtStage<S, BX, BY, VX, M, TT, MI, s> G;
+    constexpr int W0 = TbRtWarp0<S, BX, BY, VX, M, TT, MI, s>::value;
+    if (done || warp < W0 || warp >= W0 + G::W) return;
+    done = true;
+    constexpr bool XOVER = C::XOFF - G::TXL + G::NTX * VX > C::LX;
+    const int t = tid - 32 * W0;
+    const bool act = t < G::NT;
+    const int gx0 = xb - G::TXL + (t % G::NTX) * VX;
+    const int gy0 = yb - G::HY0 + (t / G::NTX) * MI;
+    const int lb = (gy0 - Y0) * C::LX + (gx0 - X0);
+    const int ry1 = yb + BY * M + G::HY1;
+    // rows: bit m = writable (inside R_s rows and the array), bit 8+m = inside the update box
+    unsigned rows = 0, allup = 1;
+#pragma unroll
+    for (int m = 0; m < MI; ++m) {
+      const int gy = gy0 + m;
+      const bool wr = gy < ry1 && gy >= 0 && gy < g.ny;
+      const bool up = gy < ry1 && gy >= g.uy0 && gy < g.uy1;
+      rows |= (wr ? 1u << m : 0u) | (up ? 1u << (8 + m) : 0u);
+      allup &= (gy >= ry1 || up) ? 1u : 0u;
+    }
+    const bool xfast = gx0 >= g.ux0 && gx0 + VX <= g.ux1 && (!XOVER || gx0 + VX <= X0 + C::LX);
+    const bool fast = act && xfast && allup;
+    unsigned long long* fin = s == 1 ? full_in : full_s(s - 1);
+    unsigned long long* ein = s == 1 ? empty_in : empty_s(s - 1);
+    constexpr int DIN = s == 1 ? NS : 2;
+    T acc[NZ][MI][VX];
+#pragma unroll
+    for (int q = 0; q < NZ; ++q) zero_acc<T, VX, MI>(acc[q]);
+#pragma unroll 1
+    for (int jb = 0; jb < nin; jb += NZ) {
+      static_for<0, NZ>([&](auto ic) {
+        constexpr int U = decltype(ic)::value;
+        const int j = jb + U;
+        if (j >= nin) return;
+        const int si = j % DIN;
+        const T* src = s == 1 ? ring0 + si * C::PLANE : mid + (2 * (s - 2) + si) * C::PLANE;
+        mbar_wait_sleep(&fin[si], (unsigned)((j / DIN) & 1));
+        zero_acc<T, VX, MI>(acc[U]);                     // a new output plane starts
+        if (act) {
+          SmemPlane<T, VX, C::LX> pl{src + lb};
+          run_scatter_ops<S, typename S::Mid, VX, MI, U>(pl, acc);
+        }
+        mbar_arrive(&ein[si]);                           // input slot read
+        const int so = j & 1;
+        T* dst = mid + (2 * (s - 1) + so) * C::PLANE;
+        if (j >= 2) mbar_wait_sleep(&empty_s(s)[so], (unsigned)((j / 2 - 1) & 1));
+        const int zo = pin0 + j - s * S::ZHI;            // plane completed now
+        const bool zin = zo >= 0 && zo < g.nz;
+        const bool zupd = zo >= g.uz0 && zo < g.uz1;
+        const T(&res)[MI][VX] = acc[(U + 1) % NZ];
+        if (zupd && fast) {                              // interior: vector stores (don't-care
+#pragma unroll                                          // values past R_s stay in the buffer)
+          for (int m = 0; m < MI; ++m)
+            if (rows & (1u << m)) stg_vec<T, VX>(dst + lb + m * C::LX, res[m]);
+        } else if (zin && act) {                         // frame / edge tiles
+#pragma unroll
+          for (int m = 0; m < MI; ++m) {
+            if (!(rows & (1u << m))) continue;
+            const bool rowupd = zupd && (rows & (1u << (8 + m)));
+            T* d = dst + lb + m * C::LX;
+            if (rowupd && xfast) {
+              stg_vec<T, VX>(d, res[m]);
+            } else {
+              const T* frame = in + (i64)zo * g.sz + (i64)(gy0 + m) * g.sy;
+#pragma unroll
+              for (int v = 0; v < VX; ++v) {
+                const int gx = gx0 + v;
+                if (gx < 0 || gx >= g.nx || gx - X0 >= C::LX) continue;
+                const bool upd = rowupd && gx >= g.ux0 && gx < g.ux1;
+                d[v] = upd ? res[m][v] : __ldg(frame + gx);
+              }
+            }
+          }
+        }
+        mbar_arrive(&full_s(s)[so]);                     // stage-s plane written
+      });
+    }
+  });
+  if (done) return;
+
+  // ------------------------------------------------------------ last stage
+  {
+    const int q = tid - 32 * C::WL;
+    const bool act = q < C::FT;
+    const int tx = q % (BX / VX), ty = q / (BX / VX);
+    const int row0 = TT * S::YLO + (CM ? ty : ty * M);
+    const int col0 = C::XOFF + tx * VX;
+    const int x0 = xb + tx * VX;
+    const int y0 = yb + (CM ? ty : ty * M);
+    unsigned long long* fin = full_s(TT - 1);
+    unsigned long long* ein = empty_s(TT - 1);
+    T acc[NZ][M][VX];
+#pragma unroll
+    for (int u = 0; u < NZ; ++u) zero_acc<T, VX, M>(acc[u]);
+#pragma unroll 1
+    for (int jb = 0; jb < nin; jb += NZ) {
+      static_for<0, NZ>([&](auto ic) {
+        constexpr int U = decltype(ic)::value;
+        const int j = jb + U;
+        if (j >= nin) return;
+        const int si = j & 1;
+        mbar_wait_sleep(&fin[si], (unsigned)((j >> 1) & 1));
+        zero_acc<T, VX, M>(acc[U]);
+        if (act) {
+          SmemPlane<T, VX, C::LX> pl{mid + (2 * (TT - 2) + si) * C::PLANE + row0 * C::LX + col0};
+          run_scatter<S, VX, M, U>(pl, acc);
+        }
+        mbar_arrive(&ein[si]);
+        const int z = pin0 + j - TT * S::ZHI;
+        if (act && z >= zs) store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc[(U + 1) % NZ]);
+      });
     }
   }
 }

@@ -129,6 +129,12 @@ static void default_params(uint32_t oc, int ndim, int dtype, stencil_params_t* p
     // (measured on C2: 128x2 fp64 tiles reach 92% of the copy bandwidth)
     p->vx = vmax; p->bx = 64 * vmax; p->by = 2; p->bz = 1;
     if (oc & STENCIL_OC_PR) p->pr_stages = 3;
+  } else if (oc & STENCIL_OC_RT) {
+    // warp-specialised retiming pipeline (k_stream_tb_rt); measured on C2:
+    // 64 x 32-row output tiles (8 threads x merge 4 rows), 3 planes in flight
+    p->vx = vmax; p->bx = 32 * vmax; p->by = 8; p->bz = 1;
+    if (merge) p->merge = 4;
+    if (oc & STENCIL_OC_PR) p->pr_stages = 3;
   } else {
     p->vx = vmax; p->bx = 32 * vmax; p->by = merge ? 4 : 8; p->bz = 1;
   }
@@ -265,7 +271,8 @@ static int resolve_variant(stencil_plan_s* P) {
             v.by, v.bz, v.m, v.vx);
   if (v.m > 8) SM_FAIL(STENCIL_E_INVAL, "merge factor must be <= 8");
   if (v.tt < 1 || v.tt > 8) SM_FAIL(STENCIL_E_INVAL, "tb_steps must be in 1..8");
-  if (v.ns < 1 || v.ns > 4) SM_FAIL(STENCIL_E_INVAL, "pr_stages must be in 1..4");
+  if (v.ns < 1 || v.ns > 8) SM_FAIL(STENCIL_E_INVAL, "pr_stages must be in 1..8");
+  if (fam == FAM_STREAM_TB && v.rt && v.tt >= 2) v.ws_threads = v.tbrt_threads(P->pat, elem);
   const int thr = v.threads();
   if (thr < 32 || thr > 1024)
     SM_FAIL(STENCIL_E_OC_INFEASIBLE, "CTA of %d threads outside 32..1024", thr);
@@ -417,6 +424,7 @@ static int launch_sweep(stencil_plan_s* P, const Variant& v, const Kernel& k, co
     gx = (g.cx1 - xa + v.bx - 1) / v.bx;
     gy = (cylen + v.by * v.m - 1) / (v.by * v.m);
     bx = v.bx / v.vx; by = v.by;
+    if (v.family == FAM_STREAM_TB && v.rt) { bx = v.threads(); by = 1; }   // warp-specialised, 1-D
     if (v.tma) SM_TRY(get_tmap(P, v, src, &tm));
     if (v.family == FAM_TILED) {
       gz = (czlen + v.bz - 1) / v.bz;
@@ -458,6 +466,10 @@ static int get_tb_rem_kernel(stencil_plan_s* P, int tt, Variant* vout, Kernel* k
   v.tt = tt;
   if (v.family == FAM_STREAM_TB && tt == 1) v.family = FAM_STREAM;   // remainder of one step: plain ST
   const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+  if (v.family == FAM_STREAM_TB && v.rt) {
+    v.ws_threads = v.tbrt_threads(P->pat, elem);
+    if (v.ws_threads > 1024) SM_FAIL(STENCIL_E_OC_INFEASIBLE, "TB remainder CTA of %d threads", v.ws_threads);
+  }
   if (v.family == FAM_TILED && v.tma) {
     const TmaBox b = tma_box(v, P->pat, elem);
     v.tma = b.lx <= 256 && b.ly <= 256 && b.lz <= 256;

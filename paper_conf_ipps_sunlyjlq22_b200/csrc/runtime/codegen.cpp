@@ -109,14 +109,19 @@ std::string Variant::name_expr(const char* desc) const {
                rt ? "true" : "false", ns, tf);
       break;
     default:
-      snprintf(b, sizeof b, "smart::k_stream_tb<%s, %d, %d, %d, %d, %s, %s, %d, %d>", desc, bx, by, vx, m,
-               cmf, rt ? "true" : "false", ns, tt);
+      if (rt)   // retiming in every fused step (k_stream_tb_rt)
+        snprintf(b, sizeof b, "smart::k_stream_tb_rt<%s, %d, %d, %d, %d, %s, %d, %d>", desc, bx, by, vx, m, cmf,
+                 ns, tt);
+      else
+        snprintf(b, sizeof b, "smart::k_stream_tb<%s, %d, %d, %d, %d, %s, %s, %d, %d>", desc, bx, by, vx, m,
+                 cmf, rt ? "true" : "false", ns, tt);
       break;
   }
   return b;
 }
 
 int Variant::threads() const {
+  if (family == FAM_STREAM_TB && rt) return ws_threads;
   switch (family) {
     case FAM_NAIVE: return bx * by;
     default: return (bx / vx) * by;
@@ -125,8 +130,32 @@ int Variant::threads() const {
 
 static int roundup(int a, int b) { return (a + b - 1) / b * b; }
 
-// rows of an intermediate-stage thread tile in k_stream_tb (S::MI)
-static constexpr int kMidRows = 2;
+// Rows of an intermediate-stage thread tile of k_stream_tb / k_stream_tb_rt
+// (S::MI). 2 rows: measured on C2 (512^3 heat, fp64), 4-row tiles of the
+// retiming pipeline need ~95 registers and lose 15% to the lower occupancy.
+int Variant::mid_rows(const Pattern& p, int elem) const {
+  (void)p; (void)elem;
+  if (family == FAM_STREAM_TB && rt)
+    if (const char* e = getenv("STENCIL_MID_ROWS")) return atoi(e);   // dev override
+  return 2;
+}
+
+// Mirrors StreamTbRtCfg::THREADS of stencil_kernels.cuh: one producer warp,
+// ceil(NT_s / 32) warps per intermediate stage s, ceil(tiles / 32) last-stage warps.
+int Variant::tbrt_threads(const Pattern& p, int elem) const {
+  const int mi = mid_rows(p, elem);
+  int warps = 1;
+  for (int s = 1; s < tt; ++s) {
+    const int hx0 = (tt - s) * p.xlo, hx1 = (tt - s) * p.xhi;
+    const int hy0 = (tt - s) * p.ylo, hy1 = (tt - s) * p.yhi;
+    const int txl = roundup(hx0, vx);
+    const int ntx = (txl + bx + hx1 + vx - 1) / vx;
+    const int nty = (by * m + hy0 + hy1 + mi - 1) / mi;
+    warps += (ntx * nty + 31) / 32;
+  }
+  warps += ((bx / vx) * by + 31) / 32;
+  return 32 * warps;
+}
 
 // Mirrors TiledCfg / StreamCfg of stencil_kernels.cuh.
 int Variant::smem_bytes(const Pattern& p, int elem) const {
@@ -148,6 +177,15 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     const int nring = (rt ? 1 : nz) + ns - 1;
     return nring * plane * elem + 8 * nring + 128;
   }
+  if (family == FAM_STREAM_TB && rt) {   // mirrors StreamTbRtCfg
+    const int xoff = roundup(tt * p.xlo, aln);
+    const int lx = roundup(xoff + bx + tt * p.xhi, aln);
+    const int ly = by * m + tt * (p.ylo + p.yhi);
+    const int plane = roundup(lx * ly * elem, 128) / elem;
+    const int padf = 128 / elem;
+    const int padb = roundup((mid_rows(p, elem) * lx + aln) * elem, 128) / elem;
+    return (padf + (ns + 2 * (tt - 1)) * plane + padb) * elem + 8 * (2 * ns + 4 * (tt - 1)) + 128;
+  }
   if (family == FAM_STREAM_TB) {   // mirrors StreamTbCfg
     const int xoff = roundup(tt * p.xlo, aln);
     const int lx = roundup(xoff + bx + tt * p.xhi, aln);
@@ -156,7 +194,7 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     const int nz = p.zlo + p.zhi + 1;
     const int nin = nz + ns - 1;
     const int padf = 128 / elem;
-    const int padb = roundup((kMidRows * lx + aln) * elem, 128) / elem;
+    const int padb = roundup((mid_rows(p, elem) * lx + aln) * elem, 128) / elem;
     return (padf + (nin + (tt - 1) * nz) * plane + padb) * elem + 8 * nin + 128;
   }
   return 0;
@@ -259,9 +297,10 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   if (ops.empty()) o << "0u";
   o << "};\n";
   std::vector<uint32_t> mops;
-  if (v.family == FAM_STREAM_TB) {     // intermediate fused steps: gather, VX x kMidRows tiles
+  const int mi = v.mid_rows(pat, f32 ? 4 : 8);
+  if (v.family == FAM_STREAM_TB) {     // intermediate fused steps: VX x MI tiles, gather or (RT) scatter
     Variant vm = v;
-    vm.family = FAM_STREAM; vm.rt = false; vm.cm = false; vm.m = kMidRows;
+    vm.family = FAM_STREAM; vm.cm = false; vm.m = mi;
     mops = encode_ops(pat, vm);
   }
   o << "__device__ constexpr unsigned g_mops[" << std::max<size_t>(mops.size(), 1) << "] = {";
@@ -269,7 +308,10 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   if (mops.empty()) o << "0u";
   o << "};\n";
   o << "struct S {\n  typedef " << T << " T;\n";
-  o << "  static constexpr int MI = " << kMidRows << ";\n";
+  o << "  static constexpr int MI = " << mi << ";\n";
+  int minb = 1;   // __launch_bounds__ min blocks of k_stream_tb_rt
+  if (const char* e = getenv("STENCIL_MINB")) minb = atoi(e);   // dev override
+  o << "  static constexpr int MINB = " << minb << ";\n";
   o << "  struct Mid {\n    static constexpr int NOPS = " << mops.size() << ";\n"
     << "    static __device__ __forceinline__ constexpr unsigned op(int i) { return g_mops[i]; }\n  };\n";
   o << "  static constexpr int NNZ = " << pat.nnz << ", ZLO = " << pat.zlo << ", ZHI = " << pat.zhi

@@ -81,9 +81,12 @@ struct Variant {
   int ns = 1;
   bool tma = false;
   int chunk = 0;         // runtime argument (streaming)
+  int ws_threads = 0;    // warp-specialised ST_TB_RT kernel: CTA size (tbrt_threads)
   std::string name_expr(const char* desc) const;
   int threads() const;
   int smem_bytes(const Pattern& p, int elem) const;
+  int mid_rows(const Pattern& p, int elem) const;
+  int tbrt_threads(const Pattern& p, int elem) const;
 };
 
 // Compiled module cache (per process): key = generated source.

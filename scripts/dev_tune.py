@@ -34,6 +34,10 @@ res = []
 for ocn in a.ocs.split(","):
     for vals in itertools.product(*[grid[k] for k in keys]):
         prm = dict(zip(keys, vals))
+        for k in list(prm):           # "env:MINB": 3 -> STENCIL_MINB=3 for this plan's codegen
+            if k.startswith("env:"):
+                os.environ["STENCIL_" + k[4:]] = str(prm.pop(k))
+        shown = dict(zip(keys, vals))
         try:
             p = sm.Plan(dims, acc, c, dtype, ocn, prm)
             p.run(x, y, a.steps)
@@ -49,8 +53,8 @@ for ocn in a.ocs.split(","):
             continue
         pts = p.info["points"]
         gs = pts * a.steps / (best * 1e-3) / 1e9
-        res.append((gs, ocn, prm, p.info["regs"], p.info["smem_bytes"]))
-        print(f"{ocn:14s} {gs:7.1f} GSt/s {gs * 2 * elem:7.0f} GB/s regs={p.info['regs']} smem={p.info['smem_bytes']} {prm}",
+        res.append((gs, ocn, shown, p.info["regs"], p.info["smem_bytes"]))
+        print(f"{ocn:14s} {gs:7.1f} GSt/s {gs * 2 * elem:7.0f} GB/s regs={p.info['regs']} smem={p.info['smem_bytes']} {shown}",
               flush=True)
         del p
 res.sort(key=lambda r: -r[0])

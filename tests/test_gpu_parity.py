@@ -216,3 +216,33 @@ def test_full_size_sampled(gpu, cfg, ocs):
         del p
     del x, y
     torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("name,dims,dtype", [("heat3d", (41, 37, 70), "f64"), ("random3d:2:5", (29, 31, 44), "f64"),
+                                             ("star25", (36, 30, 72), "f32"), ("box125", (26, 28, 40), "f64")])
+def test_tb_rt_pipeline_settings(gpu, name, dims, dtype):
+    """Warp-specialised ST_TB_RT pipeline (k_stream_tb_rt): fused depths 2..4,
+    several z-chunks per column (stream_chunk), merge modes, prefetch depths
+    1..4, and a step count that leaves a TB remainder launch."""
+    acc, c = si.config_stencil(name)
+    steps = 5
+    u0 = si.make_field(dims, 21, dtype)
+    ref = oracle.sweep(u0, acc, c, steps, dtype=dtype)
+    base = _run(sm.Plan(dims, acc, c, dtype, 0), u0, dtype, steps)
+    settings = [("ST_TB_RT", {"tb_steps": 2, "stream_chunk": 8}),
+                ("ST_TB_RT_PR", {"tb_steps": 3, "pr_stages": 4, "stream_chunk": 16}),
+                ("ST_TB_BM_RT_PR", {"tb_steps": 4, "merge": 2, "pr_stages": 2}),
+                ("ST_TB_CM_RT", {"tb_steps": 2, "merge": 4, "by": 4}),
+                ("ST_TB_BM_RT", {"tb_steps": 3, "merge": 8, "by": 2, "bx": 32})]
+    ran = 0
+    for oc, prm in settings:
+        try:
+            p = sm.Plan(dims, acc, c, dtype, sm.oc_from_name(oc), prm)
+        except sm.StencilError as e:
+            assert e.code == -3, (oc, prm, str(e))
+            continue
+        got = _run(p, u0, dtype, steps)
+        assert _relerr(got, ref) <= TOL[dtype], (oc, prm)
+        assert np.array_equal(got, base), (oc, prm)
+        ran += 1
+    assert ran >= 3
