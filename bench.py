@@ -57,6 +57,10 @@ WORKLOADS = {
     "C3": "C3: 3-D 25-point star (order 4), 768^3 fp32 per GPU, 10 time steps, ST/RT family swept, best OC timed",
     "C4": "C4: 3-D 125-point box (order 2), 512^3 fp64 per GPU, 10 time steps, TB vs tiling family swept",
     "C1": "C1: 2-D 5-point heat star (order 1), 256^2 fp64, 10 time steps, naive OC",
+    "C5": ("C5: random Algorithm-1 3-D stencils, one per order 1..4, 1024^3 fp64 per GPU, 4 time steps each, "
+           "all 30 OCs swept per stencil, best OC per stencil timed"),
+    "N2": ("N2 (NEXT-2): random Algorithm-1 2-D stencils, one per order 1..4, 8192^2 fp64 per GPU, 10 time "
+           "steps each, all 30 OCs swept per stencil (streaming along y), best OC per stencil timed"),
 }
 
 
@@ -119,41 +123,54 @@ class ClockSampler:
 def _config(name: str):
     import stencil_inputs as si
     C = dict(si.CONFIGS[name])
-    acc, c = si.config_stencil(C["stencil"])
+    acc, c = si.config_stencil(C["stencil"] if name not in si.WORKLOAD_STENCILS else si.WORKLOAD_STENCILS[name][0])
     return C, acc, c
 
 
+def _items(name: str):
+    """The stencils one bench step sweeps: one for C1-C4, one per order r = 1..4
+    for the multi-stencil workloads (C5 3-D, N2 2-D)."""
+    import stencil_inputs as si
+    names = si.WORKLOAD_STENCILS.get(name) or [si.CONFIGS[name]["stencil"]]
+    out = []
+    for sname in names:
+        acc, c = si.config_stencil(sname)
+        out.append({"stencil": sname, "acc": acc, "c": c})
+    return out
+
+
 def _ocs_for(name: str, sm):
-    if name == "C2":
-        return sm.oc_list()
     if name == "C3":
         return [o for o in sm.oc_list() if o & sm.OC_ST and not o & sm.OC_TB]
     if name == "C4":
         return [o for o in sm.oc_list() if not o & sm.OC_ST or o & sm.OC_RT]
     if name == "C1":
         return [0]
-    return sm.oc_list()
+    return sm.oc_list()      # C2, C5, N2: all 30 OCs
 
 
-def cpu_oracle_sample(name: str, budget_s: float = 12.0):
+def cpu_oracle_sample(name: str, budget_s: float = 12.0, acc=None, c=None):
     """Time the oracle (as it stands) on a bounded z-slab of the workload."""
     import oracle
     import stencil_inputs as si
-    C, acc, c = _config(name)
+    C, acc0, c0 = _config(name)
+    if acc is None:
+        acc, c = acc0, c0
     dims, steps, dtype = C["dims"], C["steps"], C["dtype"]
     r = (acc.shape[0] - 1) // 2
     threads = oracle.max_threads()
-    if len(dims) == 2:
+    if len(dims) == 2 and dims[0] * dims[1] <= 1 << 20:
         u = si.make_field(dims, C["seed"], dtype)
         t0 = time.perf_counter()
         oracle.sweep(u, acc, c, steps, dtype=dtype)
         dt = time.perf_counter() - t0
         pts = (dims[0] - 2 * r) * (dims[1] - 2 * r) * steps
         return {"value": pts / dt / 1e9, "unit": "GStencil/s", "cores": threads, "kind": "oracle",
-                "sample": f"full C1 grid {dims}, {steps} steps, {dt:.2f} s", "seconds": dt}
-    # probe with a thin slab, then size the sample to ~budget_s
+                "sample": f"full {name} grid {dims}, {steps} steps, {dt:.2f} s", "seconds": dt, "points": pts}
+    # probe with a thin slab (rows in 2-D, planes in 3-D), then size the sample to ~budget_s
+    row = tuple(dims[1:])
     nz = 2 * r + 8
-    u = si.make_field((nz, dims[1], dims[2]), C["seed"], dtype, global_dims=dims)
+    u = si.make_field((nz,) + row, C["seed"], dtype, global_dims=dims)
     t0 = time.perf_counter()
     oracle.sweep(u, acc, c, 1, dtype=dtype)
     per_plane = (time.perf_counter() - t0) / (nz - 2 * r)
@@ -163,14 +180,55 @@ def cpu_oracle_sample(name: str, budget_s: float = 12.0):
     else:
         s_steps = max(1, min(steps, int(budget_s / max(per_plane * full, 1e-9))))
         planes = int(max(8, min(full, budget_s / max(per_plane, 1e-9) / s_steps)))
-    u = si.make_field((planes + 2 * r, dims[1], dims[2]), C["seed"], dtype, global_dims=dims)
+    u = si.make_field((planes + 2 * r,) + row, C["seed"], dtype, global_dims=dims)
     t0 = time.perf_counter()
     oracle.sweep(u, acc, c, s_steps, dtype=dtype)
     dt = time.perf_counter() - t0
-    pts = planes * (dims[1] - 2 * r) * (dims[2] - 2 * r) * s_steps
+    inner = 1
+    for d in row:
+        inner *= d - 2 * r
+    pts = planes * inner * s_steps
+    unit = "planes" if len(dims) == 3 else "rows"
     return {"value": pts / dt / 1e9, "unit": "GStencil/s", "cores": threads, "kind": "oracle",
-            "sample": (f"{planes}+{2 * r} planes x {dims[1]}x{dims[2]} of the {name} grid, {s_steps} step(s), "
-                       f"{dt:.2f} s; rate per interior update"), "seconds": dt}
+            "sample": (f"{planes}+{2 * r} {unit} x {'x'.join(map(str, row))} of the {name} grid, {s_steps} step(s), "
+                       f"{dt:.2f} s; rate per interior update"), "seconds": dt, "points": pts}
+
+
+def _cpu_workload(name: str, budget_s: float):
+    """Oracle rate over every stencil of the workload: total sampled updates /
+    total seconds (the same aggregation as the GPU value)."""
+    items = _items(name)
+    per = budget_s / len(items)
+    samples = [cpu_oracle_sample(name, per, it["acc"], it["c"]) for it in items]
+    pts = sum(x["points"] for x in samples)
+    sec = sum(x["seconds"] for x in samples)
+    # time-weighted: each stencil's full-workload time at its sampled rate
+    C = _config(name)[0]
+    tot_pts, tot_s = 0, 0.0
+    for it, x in zip(items, samples):
+        r = (it["acc"].shape[0] - 1) // 2
+        n = 1
+        for d in C["dims"]:
+            n *= d - 2 * r
+        tot_pts += n * C["steps"]
+        tot_s += n * C["steps"] / (x["value"] * 1e9)
+    v = tot_pts / tot_s / 1e9
+    sample = "; ".join(f"{it['stencil']}: {x['sample']}" for it, x in zip(items, samples)) if len(items) > 1 \
+        else samples[0]["sample"]
+    return {"value": v, "unit": "GStencil/s", "cores": samples[0]["cores"], "kind": "oracle", "sample": sample,
+            "seconds": sec, "points": pts}
+
+
+def _workload_points(name: str) -> int:
+    C = _config(name)[0]
+    tot = 0
+    for it in _items(name):
+        r = (it["acc"].shape[0] - 1) // 2
+        n = 1
+        for d in C["dims"]:
+            n *= d - 2 * r
+        tot += n * C["steps"]
+    return tot
 
 
 def run_reference(args):
@@ -182,22 +240,19 @@ def run_reference(args):
     vals = []
     cb = None
     for i in range(args.warmup + args.steps):
-        cb = cpu_oracle_sample(name, budget)
+        cb = _cpu_workload(name, budget)
         if i >= args.warmup:
             vals.append(cb["value"])
     v = statistics.mean(vals)
-    C, acc, c = _config(name)
-    pts = 1
-    r = (acc.shape[0] - 1) // 2
-    for d in C["dims"]:
-        pts *= d - 2 * r
-    ms = pts * C["steps"] / (v * 1e9) * 1e3
+    C = _config(name)[0]
+    ms = _workload_points(name) / (v * 1e9) * 1e3
     line = {
         "impl": "reference", "metric": METRIC, "value": v, "unit": "GStencil/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": C["dtype"], "data": "synthetic",
         "config": {"workload": WORKLOADS.get(name, name), "grid": list(C["dims"]), "time_steps": C["steps"],
-                   "note": "oracle timed on a bounded z-slab sample; ms_per_step extrapolated to the full grid"},
+                   "stencils": [it["stencil"] for it in _items(name)],
+                   "note": "oracle timed on a bounded slab sample; ms_per_step extrapolated to the full grid"},
         "cpu_baseline": {k: cb[k] for k in ("kind", "cores", "sample")} | {"value": v, "unit": "GStencil/s"},
         "e2e": {"value": v, "unit": "GStencil/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
@@ -230,6 +285,40 @@ def _traffic_from_profiles(key: str):
         return None
 
 
+def _roofline(name, sm, pinfo, oc, pts, steps, kern_ms, kern_n, total_ms, nsteps_timed, elem, dtype, peak, peak_kind):
+    """Roofline of one stencil's sweep kernel: algorithmic bytes
+    per launch (read + write every interior point once) / average launch time,
+    and the FMA ceiling; the binding one is reported."""
+    T = pinfo["params"]["tb_steps"] if oc & sm.OC_TB else 1
+    groups = nsteps_timed * math.ceil(steps / T)
+    bytes_per_launch = pts * 2 * elem
+    flops_per_step = pts * 2 * pinfo["nnz"]    # one FMA per neighbour per point and step
+    avg_launch_ms = kern_ms / max(groups, 1)
+    achieved = bytes_per_launch / (avg_launch_ms * 1e-3) / 1e9
+    # DESIGN.md §6: FP64 148 SM x 64 FMA/clk x 2 x 1.965 GHz = 37.2 TFLOP/s; FP32 x2
+    fp_peak = 148 * 64 * 2 * 1.965e9 / 1e12 * (1 if dtype == "f64" else 2)
+    achieved_fp = flops_per_step * nsteps_timed * steps / (kern_ms * 1e-3) / 1e12
+    key = kernel_key(name, pinfo["kernel_name"])
+    roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+            "frac": round(achieved / peak, 4), "traffic": _traffic_from_profiles(key),
+            "peak_kind": peak_kind, "kernel": key,
+            "launch_ms": round(avg_launch_ms, 4), "launches": kern_n,
+            "kernel_share_of_step": round(kern_ms / max(total_ms, 1e-9), 4),
+            "bytes_per_launch": bytes_per_launch, "time_steps_per_launch": T,
+            "frac_of_spec_8tbs": round(achieved / HBM_SPEC_GBS, 4),
+            "fp": {"achieved": round(achieved_fp, 2), "peak": round(fp_peak, 1), "unit": "TFLOP/s",
+                   "frac": round(achieved_fp / fp_peak, 4), "peak_kind": "derived (DESIGN.md §6)"}}
+    # FMA-bound stencils (C4, high-order random): the FP ceiling binds before HBM
+    if flops_per_step / (fp_peak * 1e12) > bytes_per_launch / T / (peak * 1e9):
+        roof.update({"bound": "alu", "achieved": round(achieved_fp, 2), "peak": round(fp_peak, 1),
+                     "unit": "TFLOP/s", "frac": round(achieved_fp / fp_peak, 4),
+                     "peak_kind": "derived (DESIGN.md §6)",
+                     "hbm": {"achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                             "frac": round(achieved / peak, 4)}})
+        roof.pop("fp")
+    return roof
+
+
 def run_impl(args):
     import torch
     import torch.distributed as dist
@@ -242,16 +331,17 @@ def run_impl(args):
         dist.init_process_group("nccl", device_id=dev)
     sm.lib()
     name = args.config
-    C, acc, c = _config(name)
+    C = _config(name)[0]
     dims, steps, dtype = tuple(C["dims"]), C["steps"], C["dtype"]
     tdt = torch.float64 if dtype == "f64" else torch.float32
     elem = 8 if dtype == "f64" else 4
     peak, peak_kind = _peaks()
+    items = _items(name)
 
     slab = (world > 1 or args.slab) and len(dims) == 3
     comm_owner = []
 
-    def make_plan(oc, params=None):
+    def make_plan(acc, c, oc, params=None):
         """Plan on this rank's slab; the halo exchange (a7) runs on torch's NCCL
         communicator (N > 1) or on one library-owned communicator (N = 1)."""
         p = sm.Plan(dims, acc, c, dtype, oc, params)
@@ -267,12 +357,13 @@ def run_impl(args):
         return p
 
     # every rank owns dims[0] planes of a global grid of depth world*dims[0]
-    # (weak scaling); slab buffers carry G ghost planes on each side
-    base_plan = make_plan(0)
-    info0 = base_plan.info
-    G = base_plan.ghost
+    # (weak scaling); slab buffers carry G ghost planes on each side. One
+    # input/output pair (and one workspace) serves every stencil of the step.
+    probe = make_plan(items[0]["acc"], items[0]["c"], 0)
+    G = probe.ghost
+    shape = probe.array_shape
     gdims = (dims[0] * world,) + dims[1:] if len(dims) == 3 else dims
-    x = torch.zeros(base_plan.array_shape, dtype=tdt, device=dev)
+    x = torch.zeros(shape, dtype=tdt, device=dev)
     if len(dims) == 3:
         z0 = dims[0] * rank
         a, b = max(0, z0 - G), min(gdims[0], z0 + dims[0] + G)
@@ -280,72 +371,88 @@ def run_impl(args):
     else:
         sm.fill_field(x, C["seed"], 0)
     y = torch.empty_like(x)
+    ws = torch.empty(probe.workspace_bytes() // elem, dtype=tdt, device=dev)
+    del probe
     stream = torch.cuda.current_stream()
 
-    # ---- 1. label pass: every OC of the family, seeded settings (a8)
-    pts = info0["points"]                      # this rank's interior points per time step
-    pts_all = pts
-    if world > 1:
-        t = torch.tensor([pts], dtype=torch.float64, device=dev)
-        dist.all_reduce(t)
-        pts_all = int(t.item())
+    # ---- 1. label pass per stencil: every OC of the family, seeded settings (a8)
     ocs = _ocs_for(name, sm)
     if args.oc:
         ocs = [sm.oc_from_name(args.oc)]
     t_sw = time.time()
-    if args.settings > 0 and len(ocs) > 1:
-        sweep = base_plan.oc_sweep(x, y, steps=steps, settings_per_oc=args.settings, reps=3, seed=args.seed)
-    else:
-        sweep = {"oc_ids": sm.oc_list(), "times_ms": [math.inf] * sm.NUM_OC,
-                 "best_params": [{}] * sm.NUM_OC, "best_oc": ocs[0]}
+    for it in items:
+        base_plan = make_plan(it["acc"], it["c"], 0)
+        base_plan.use_workspace(ws)
+        info0 = base_plan.info
+        it["points"] = info0["points"]          # this rank's interior points per time step
+        it["nnz"] = info0["nnz"]
+        if args.settings > 0 and len(ocs) > 1:
+            sweep = base_plan.oc_sweep(x, y, steps=steps, settings_per_oc=args.settings, reps=3, seed=args.seed)
+        else:
+            sweep = {"oc_ids": sm.oc_list(), "times_ms": [math.inf] * sm.NUM_OC,
+                     "best_params": [{}] * sm.NUM_OC, "best_oc": ocs[0]}
+        per_oc, best_oc, best_t, best_p = {}, None, math.inf, None
+        for oc, t, p in zip(sweep["oc_ids"], sweep["times_ms"], sweep["best_params"]):
+            if oc not in ocs:
+                continue
+            gs = sm.gstencil_per_s(it["points"], steps, t) if math.isfinite(t) else None
+            per_oc[sm.oc_name(oc)] = {
+                "ms": round(t, 4) if math.isfinite(t) else None,
+                "gstencil_s": round(gs, 2) if gs else None,
+                "hbm_frac_of_measured": round(gs * 2 * elem / peak, 4) if gs else None,
+                "hbm_frac_of_spec": round(gs * 2 * elem / HBM_SPEC_GBS, 4) if gs else None,
+                "infeasible": not math.isfinite(t),
+            }
+            if math.isfinite(t) and t < best_t:
+                best_oc, best_t, best_p = oc, t, p
+        if best_oc is None:
+            best_oc, best_p = ocs[0], None
+        if args.params:
+            best_p = json.loads(args.params)
+        if world > 1:   # every rank must run the same OC: take rank 0's label
+            obj = [best_oc, best_p]
+            dist.broadcast_object_list(obj, src=0)
+            best_oc, best_p = obj
+        it["per_oc"], it["best_oc"] = per_oc, best_oc
+        del base_plan
+        it["plan"] = make_plan(it["acc"], it["c"], best_oc, best_p or None)
+        it["plan"].use_workspace(ws)
+        it["pinfo"] = it["plan"].info
     sweep_s = time.time() - t_sw
-    per_oc = {}
-    best_oc, best_t, best_p = None, math.inf, None
-    for oc, t, p in zip(sweep["oc_ids"], sweep["times_ms"], sweep["best_params"]):
-        if oc not in ocs:
-            continue
-        gs = sm.gstencil_per_s(pts, steps, t) if math.isfinite(t) else None
-        per_oc[sm.oc_name(oc)] = {
-            "ms": round(t, 4) if math.isfinite(t) else None,
-            "gstencil_s": round(gs, 2) if gs else None,
-            "hbm_frac_of_measured": round(gs * 2 * elem / peak, 4) if gs else None,
-            "hbm_frac_of_spec": round(gs * 2 * elem / HBM_SPEC_GBS, 4) if gs else None,
-            "infeasible": not math.isfinite(t),
-        }
-        if math.isfinite(t) and t < best_t:
-            best_oc, best_t, best_p = oc, t, p
-    if best_oc is None:
-        best_oc, best_p = ocs[0], None
-    if args.params:
-        best_p = json.loads(args.params)
-    if world > 1:   # every rank must run the same OC: take rank 0's label
-        obj = [best_oc, best_p]
-        dist.broadcast_object_list(obj, src=0)
-        best_oc, best_p = obj
+    pts_rank = sum(it["points"] for it in items)
+    pts_all = pts_rank
+    if world > 1:
+        t = torch.tensor([pts_rank], dtype=torch.float64, device=dev)
+        dist.all_reduce(t)
+        pts_all = int(t.item())
 
-    plan = make_plan(best_oc, best_p or None)
-    pinfo = plan.info
+    def step():
+        for it in items:
+            it["plan"].run(x, y, steps)
 
-    # ---- 2. warm-up + timed steps
+    # ---- 2. warm-up + timed steps (one step = every stencil of the workload)
     for _ in range(args.warmup):
-        plan.run(x, y, steps)
+        step()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     launches0 = sm.launch_count()
-    plan.set_timing(True)
+    for it in items:
+        it["plan"].kernel_time()                   # reset the per-launch accumulators
+        it["plan"].set_timing(True)
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         e0.record(stream)
         for _ in range(args.steps):
-            plan.run(x, y, steps)
+            step()
         e1.record(stream)
         torch.cuda.synchronize()
     launches = sm.launch_count() - launches0
-    kern_ms, kern_n = plan.kernel_time()
-    plan.set_timing(False)
+    for it in items:
+        it["kern_ms"], it["kern_n"] = it["plan"].kernel_time()
+        it["plan"].set_timing(False)
     total_ms = e0.elapsed_time(e1)
     if world > 1:
         t = torch.tensor([total_ms], device=dev)
@@ -355,35 +462,14 @@ def run_impl(args):
     ms_per_step = total_ms / args.steps
     value = pts_all * steps / (ms_per_step * 1e-3) / 1e9
 
-    # ---- 3. roofline of the dominant kernel (the labelled OC's sweep kernel)
-    # A "launch" here is one application of the kernel to the whole owned grid
-    # (with slabs it is split into edge + interior pieces; their times add up).
-    T = pinfo["params"]["tb_steps"] if best_oc & sm.OC_TB else 1
-    groups = args.steps * math.ceil(steps / T)
-    bytes_per_launch = pts * 2 * elem          # read + write each interior point once per launch
-    flops_per_step = pts * 2 * pinfo["nnz"]    # one FMA per neighbour per point and step
-    avg_launch_ms = kern_ms / max(groups, 1)
-    achieved = bytes_per_launch / (avg_launch_ms * 1e-3) / 1e9
-    # FP64 148 SM x 64 FMA/clk x 2 x 1.965 GHz = 37.2 TFLOP/s; FP32 x2
-    fp_peak = 148 * 64 * 2 * 1.965e9 / 1e12 * (1 if dtype == "f64" else 2)
-    achieved_fp = flops_per_step * args.steps * steps / (kern_ms * 1e-3) / 1e12
-    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(achieved / peak, 4),
-                "traffic": _traffic_from_profiles(kernel_key(name, pinfo["kernel_name"])),
-                "peak_kind": peak_kind, "kernel": kernel_key(name, pinfo["kernel_name"]),
-                "launch_ms": round(avg_launch_ms, 4), "launches": kern_n,
-                "kernel_share_of_step": round(kern_ms / max(total_ms, 1e-9), 4),
-                "bytes_per_launch": bytes_per_launch, "time_steps_per_launch": T,
-                "frac_of_spec_8tbs": round(achieved / HBM_SPEC_GBS, 4),
-                "fp": {"achieved": round(achieved_fp, 2), "peak": round(fp_peak, 1), "unit": "TFLOP/s",
-                       "frac": round(achieved_fp / fp_peak, 4), "peak_kind": "derived (DESIGN.md §6)"}}
-    if achieved_fp / fp_peak > achieved / peak:   # FMA-bound stencil (C4, high-order random)
-        roofline.update({"bound": "alu", "achieved": round(achieved_fp, 2), "peak": round(fp_peak, 1),
-                         "unit": "TFLOP/s", "frac": round(achieved_fp / fp_peak, 4),
-                         "peak_kind": "derived (DESIGN.md §6)",
-                         "hbm": {"achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                                 "frac": round(achieved / peak, 4)}})
-        roofline.pop("fp")
+    # ---- 3. roofline per stencil; the dominant kernel (largest share of the step) is reported
+    for it in items:
+        it["roofline"] = _roofline(name, sm, it["pinfo"], it["best_oc"], it["points"], steps, it["kern_ms"],
+                                   it["kern_n"], total_ms, args.steps, elem, dtype, peak, peak_kind)
+    dom = max(items, key=lambda it: it["kern_ms"])
+    roofline = dict(dom["roofline"])
+    if len(items) > 1:
+        roofline["stencil"] = dom["stencil"]
 
     # ---- 4. e2e through the public API with host buffers
     e2e = None
@@ -391,19 +477,21 @@ def run_impl(args):
         hin = torch.empty(tuple(x.shape), dtype=tdt, pin_memory=True)
         hin.copy_(x.cpu())
         hout = torch.empty_like(hin).pin_memory()
-        plan.run_host(hin, hout, steps)   # warm (allocates the plan's device buffers)
+        for it in items:
+            it["plan"].run_host(hin, hout, steps)   # warm (allocates the plan's device buffers)
         n_e2e = max(1, min(3, args.steps))
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         for _ in range(n_e2e):
-            plan.run_host(hin, hout, steps)
+            for it in items:
+                it["plan"].run_host(hin, hout, steps)
         torch.cuda.synchronize()
         e2e_ms = (time.perf_counter() - t0) * 1e3 / n_e2e
         if world > 1:
             t = torch.tensor([e2e_ms], device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e2e_ms = float(t.item())
-        nbytes = x.numel() * elem
+        nbytes = x.numel() * elem * len(items)
         e2e = {"value": round(pts_all * steps / (e2e_ms * 1e-3) / 1e9, 3), "unit": "GStencil/s",
                "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes, "ms_per_step": round(e2e_ms, 3)}
         del hin, hout
@@ -411,10 +499,11 @@ def run_impl(args):
     # ---- 5. CPU oracle beside it (rank 0, N = 1)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
-        cb = cpu_oracle_sample(name, args.cpu_budget)
+        cb = _cpu_workload(name, args.cpu_budget)
         cpu = {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample")}
 
     if rank == 0:
+        first = items[0]
         line = {
             "metric": METRIC, "value": round(value, 2), "unit": "GStencil/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4),
@@ -422,7 +511,11 @@ def run_impl(args):
             "data": "synthetic",
             "config": {"workload": WORKLOADS.get(name, name), "grid_per_gpu": list(dims),
                        "global_grid": list(gdims), "time_steps_per_step": steps,
-                       "stencil": C["stencil"], "oc": sm.oc_name(best_oc), "params": pinfo["params"],
+                       "stencil": first["stencil"] if len(items) == 1 else [it["stencil"] for it in items],
+                       "oc": sm.oc_name(first["best_oc"]) if len(items) == 1
+                       else {it["stencil"]: sm.oc_name(it["best_oc"]) for it in items},
+                       "params": first["pinfo"]["params"] if len(items) == 1
+                       else {it["stencil"]: it["pinfo"]["params"] for it in items},
                        "parallelism": (f"z-slabs x{world}, NCCL halo exchange (ghost {G} planes), edge/interior overlap"
                                        if slab else "single GPU"),
                        "l2": "inputs (grid bytes) larger than the 126 MB L2; no flush needed"},
@@ -433,10 +526,19 @@ def run_impl(args):
             "e2e": e2e,
             "gpu_launches": launches,
             "clocks": clk.result(),
-            "best_oc": sm.oc_name(best_oc),
-            "per_oc": per_oc,
+            "best_oc": sm.oc_name(first["best_oc"]) if len(items) == 1
+            else {it["stencil"]: sm.oc_name(it["best_oc"]) for it in items},
+            "per_oc": first["per_oc"] if len(items) == 1 else {it["stencil"]: it["per_oc"] for it in items},
             "label_sweep": {"settings_per_oc": args.settings, "reps": 3, "seconds": round(sweep_s, 1)},
         }
+        if len(items) > 1:
+            line["stencils"] = [{
+                "stencil": it["stencil"], "order": (it["acc"].shape[0] - 1) // 2, "nnz": it["nnz"],
+                "best_oc": sm.oc_name(it["best_oc"]),
+                "gstencil_s": round(it["points"] * steps * args.steps / (it["kern_ms"] * 1e-3) / 1e9, 2)
+                if it["kern_ms"] > 0 else None,
+                "roofline": {k: it["roofline"][k] for k in ("bound", "achieved", "peak", "unit", "frac")}}
+                for it in items]
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.barrier()
@@ -450,8 +552,9 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4"])
-    ap.add_argument("--settings", type=int, default=2, help="settings per OC in the label pass")
+    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5", "N2"])
+    ap.add_argument("--settings", type=int, default=None,
+                    help="settings per OC in the label pass (default 2; 1 for the multi-stencil C5/N2)")
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--oc", default="", help="time this OC (skips the label pass); for profiling")
     ap.add_argument("--params", default="", help="JSON parameter setting for --oc")
@@ -462,6 +565,8 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
+    if args.settings is None:
+        args.settings = 1 if args.config in ("C5", "N2") else 2
     if args.impl == "reference":
         return run_reference(args)
     return run_impl(args)

@@ -351,6 +351,14 @@ class Plan:
             _check(lib().stencil_plan_set_workspace(self._h, ctypes.c_void_p(self._ws.data_ptr()),
                                                     self.workspace_bytes()))
 
+    def use_workspace(self, t) -> None:
+        """Use a caller-owned device tensor (>= workspace_bytes()) as the ping-pong
+        workspace, e.g. one workspace shared by several plans of the same shape."""
+        if t.numel() * t.element_size() < self.workspace_bytes():
+            raise ValueError("workspace tensor too small")
+        self._ws = t
+        _check(lib().stencil_plan_set_workspace(self._h, ctypes.c_void_p(t.data_ptr()), self.workspace_bytes()))
+
     @property
     def ghost(self) -> int:
         """Ghost planes on each side of the slab (0 without a communicator)."""

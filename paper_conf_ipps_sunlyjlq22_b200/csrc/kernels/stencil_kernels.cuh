@@ -283,6 +283,46 @@ __device__ __forceinline__ void store_tile(T* __restrict__ out, const Grid& g, i
   }
 }
 
+// The same store with the plane-invariant part hoisted: streaming kernels
+// build it once per thread and store one tile per plane.
+template <class T, int VX, int M, bool CM, int BYS>
+struct TileStore {
+  T* base;             // element (plane 0, row y0, column x0)
+  i64 sz, rs;          // plane stride, stride between the tile's rows
+  unsigned rows;       // bit m: row m inside the compute box
+  bool full;           // whole vectors inside the compute box (128-bit stores)
+  int x0, cx0, cx1;
+  __device__ __forceinline__ TileStore(T* out, const Grid& g, int y0, int x0_) {
+    x0 = x0_; cx0 = g.cx0; cx1 = g.cx1;
+    base = out + (i64)y0 * g.sy + x0;
+    sz = g.sz;
+    rs = (CM ? BYS : 1) * g.sy;
+    full = (x0 >= g.cx0) && (x0 + VX <= g.cx1) && g.vec_ok;
+    rows = 0;
+#pragma unroll
+    for (int m = 0; m < M; ++m) {
+      const int y = CM ? y0 + m * BYS : y0 + m;
+      if (y >= g.cy0 && y < g.cy1) rows |= 1u << m;
+    }
+  }
+  __device__ __forceinline__ void store(int z, const T (&acc)[M][VX]) const {
+    T* p = base + (i64)z * sz;
+    if (full) {
+#pragma unroll
+      for (int m = 0; m < M; ++m)
+        if (rows & (1u << m)) stg_vec<T, VX>(p + m * rs, acc[m]);
+    } else {
+#pragma unroll
+      for (int m = 0; m < M; ++m) {
+        if (!(rows & (1u << m))) continue;
+#pragma unroll
+        for (int v = 0; v < VX; ++v)
+          if (x0 + v >= cx0 && x0 + v < cx1) p[m * rs + v] = acc[m][v];
+      }
+    }
+  }
+};
+
 template <class T, int VX, int M>
 __device__ __forceinline__ void zero_acc(T (&acc)[M][VX]) {
 #pragma unroll
@@ -551,6 +591,7 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
   const int col0 = C::XOFF + tx * VX;
   const int x0 = xb + tx * VX;
   const int y0 = yb + (CM ? ty : ty * M);
+  const TileStore<T, VX, M, CM, BY> ts(out, g, y0, x0);
 
   if constexpr (RT) {
     T acc[NZ][M][VX];
@@ -570,7 +611,7 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
           SmemPlane<T, VX, C::LX> pl{ring + (it % C::NRING) * C::PLANE + row0 * C::LX + col0};
           run_scatter<S, VX, M, U>(pl, acc);
           const int z = pfirst + it - S::ZHI;             // output completed by this plane
-          if (z >= zs) store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc[(U + 1) % NZ]);
+          if (z >= zs) ts.store(z, acc[(U + 1) % NZ]);
           __syncthreads();                                // slot it%NRING may be refilled
         }
       });
@@ -590,7 +631,7 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
         for (int zi = 0; zi < NZ; ++zi)                  // plane z + zi - ZLO
           pl[zi].p = ring + ((it - (NZ - 1) + zi) % C::NRING) * C::PLANE + row0 * C::LX + col0;
         run_gather<S, VX, M>(pl, acc);
-        store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc);
+        ts.store(z, acc);
       }
       __syncthreads();                                    // oldest slot may be refilled
     }
@@ -1029,6 +1070,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     const int col0 = C::XOFF + tx * VX;
     const int x0 = xb + tx * VX;
     const int y0 = yb + (CM ? ty : ty * M);
+    const TileStore<T, VX, M, CM, BY> ts(out, g, y0, x0);
     unsigned long long* fin = full_s(TT - 1);
     unsigned long long* ein = empty_s(TT - 1);
     T acc[NZ][M][VX];
@@ -1049,7 +1091,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         }
         mbar_arrive(&ein[si]);
         const int z = pin0 + j - TT * S::ZHI;
-        if (act && z >= zs) store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc[(U + 1) % NZ]);
+        if (act && z >= zs) ts.store(z, acc[(U + 1) % NZ]);
       });
     }
   }

@@ -16,7 +16,7 @@ CACHE = os.path.expanduser("~/.cache/stencilmart")
 
 
 def newest_cubin():
-    fs = glob.glob(os.path.join(CACHE, "*.cubin"))
+    fs = glob.glob(os.path.join(os.environ.get("STENCIL_CACHE_DIR", CACHE), "*.cubin"))
     return max(fs, key=os.path.getmtime) if fs else None
 
 
@@ -30,7 +30,9 @@ for spec in sys.argv[1:]:
     sname = name.replace("-", ":")
     acc, c = si.config_stencil(sname)
     dims = (64, 64, 64) if acc.ndim == 3 else (256, 256)
-    before = newest_cubin()
+    import tempfile
+    CACHE = tempfile.mkdtemp(prefix="smcc")
+    os.environ["STENCIL_CACHE_DIR"] = CACHE
     try:
         p = sm.Plan(dims, acc, c, dtype, sm.oc_from_name(oc), prm)
     except sm.StencilError as e:

@@ -223,10 +223,10 @@ def config_stencil(name: str, seed: int = 0):
         return star25()
     if name == "box125":
         return box125()
-    if name.startswith("random3d"):
-        # random3d:<order>:<seed>
-        _, order, s = name.split(":")
-        acc, _ = random_stencil(3, int(order), int(s))
+    if name.startswith("random3d") or name.startswith("random2d"):
+        # random{3,2}d:<order>:<seed>
+        kind, order, s = name.split(":")
+        acc, _ = random_stencil(3 if kind == "random3d" else 2, int(order), int(s))
         return acc, random_coeffs(acc, int(s))
     raise KeyError(name)
 
@@ -276,4 +276,14 @@ CONFIGS: Dict[str, dict] = {
     "C3": dict(ndim=3, dims=(768, 768, 768), stencil="star25", dtype="f32", steps=10, seed=0xC0FFEE + 3),
     "C4": dict(ndim=3, dims=(512, 512, 512), stencil="box125", dtype="f64", steps=10, seed=0xC0FFEE + 4),
     "C5": dict(ndim=3, dims=(1024, 1024, 1024), stencil="random3d", dtype="f64", steps=4, seed=0xC0FFEE + 5),
+    # NEXT-2: the paper's 2-D dataset size, 8192^2, random 2-D stencils
+    "N2": dict(ndim=2, dims=(8192, 8192), stencil="random2d", dtype="f64", steps=10, seed=0xC0FFEE + 6),
+}
+
+# The stencils a multi-stencil workload sweeps: one Algorithm-1 stencil per
+# order r = 1..4 (stencil seeds 0-15, order = 1 + seed/4;
+# the bench takes the first seed of each order).
+WORKLOAD_STENCILS: Dict[str, List[str]] = {
+    "C5": [f"random3d:{r}:{4 * (r - 1)}" for r in range(1, 5)],
+    "N2": [f"random2d:{r}:{4 * (r - 1)}" for r in range(1, 5)],
 }
