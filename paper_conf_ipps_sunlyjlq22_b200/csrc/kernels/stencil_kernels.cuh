@@ -16,6 +16,8 @@
 //   static __device__ constexpr T coef(int i);
 //   static constexpr int NOPS; static __device__ constexpr unsigned op(int i);
 //       the variant's op table (see run_gather / run_scatter).
+//   static constexpr int RTSHIFT;  1: retiming queues rotate by register
+//       shifts (one plane body) instead of NZ unrolled bodies (large tables).
 //
 // Arithmetic contract (SURVEY C-4): every output
 // is ONE fused-multiply-add chain acc = fma(c_o, u[p+o], acc) starting from 0
@@ -323,6 +325,21 @@ struct TileStore {
   }
 };
 
+// acc[d] <- acc[d+1], acc[NZ-1] <- 0 (register moves after full unrolling)
+template <class T, int NZ, int M, int VX>
+__device__ __forceinline__ void shift_queue(T (&acc)[NZ][M][VX]) {
+#pragma unroll
+  for (int d = 0; d + 1 < NZ; ++d)
+#pragma unroll
+    for (int m = 0; m < M; ++m)
+#pragma unroll
+      for (int v = 0; v < VX; ++v) acc[d][m][v] = acc[d + 1][m][v];
+#pragma unroll
+  for (int m = 0; m < M; ++m)
+#pragma unroll
+    for (int v = 0; v < VX; ++v) acc[NZ - 1][m][v] = T(0);
+}
+
 template <class T, int VX, int M>
 __device__ __forceinline__ void zero_acc(T (&acc)[M][VX]) {
 #pragma unroll
@@ -593,7 +610,27 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
   const int y0 = yb + (CM ? ty : ty * M);
   const TileStore<T, VX, M, CM, BY> ts(out, g, y0, x0);
 
-  if constexpr (RT) {
+  if constexpr (RT && S::RTSHIFT) {
+    // large op tables (high-order stencils): one copy of the plane body and a
+    // register shift of the queue per plane (NZ*M*VX moves against NNZ*M*VX
+    // FMAs) -- NZ unrolled copies would overflow the instruction cache.
+    // acc[d] = partial sums of the output plane completing d planes from now.
+    T acc[NZ][M][VX];
+#pragma unroll
+    for (int q = 0; q < NZ; ++q) zero_acc<T, VX, M>(acc[q]);
+#pragma unroll 1
+    for (int it = 0; it < nit; ++it) {
+      if (it + NS - 1 < nit) issue(it + NS - 1);
+      if constexpr (!TMA) cp_async_commit();
+      wait_plane(it);
+      SmemPlane<T, VX, C::LX> pl{ring + (it % C::NRING) * C::PLANE + row0 * C::LX + col0};
+      run_scatter<S, VX, M, NZ - 1>(pl, acc);           // slice zi -> acc[NZ-1-zi]
+      const int z = pfirst + it - S::ZHI;               // output completed by this plane
+      if (z >= zs) ts.store(z, acc[0]);
+      shift_queue<T, NZ, M, VX>(acc);
+      __syncthreads();                                  // slot it%NRING may be refilled
+    }
+  } else if constexpr (RT) {
     T acc[NZ][M][VX];
 #pragma unroll
     for (int q = 0; q < NZ; ++q) zero_acc<T, VX, M>(acc[q]);
@@ -805,14 +842,21 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
         const int q = pin0 + it - (TT - 1) * S::ZHI;
         SmemPlane<T, VX, C::LX> pl{stage_plane(TT - 1, q) + row0 * C::LX + col0};
         const int z = q - S::ZHI;
-        static_for<0, NZ>([&](auto ic) {
-          constexpr int UR = decltype(ic)::value;
-          if (ur == UR) {
-            zero_acc<T, VX, M>(acc[UR]);
-            run_scatter<S, VX, M, UR>(pl, acc);
-            if (z >= zs) store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc[(UR + 1) % NZ]);
-          }
-        });
+        if constexpr (S::RTSHIFT) {                      // one body + register shift (see k_stream)
+          (void)ur;
+          run_scatter<S, VX, M, NZ - 1>(pl, acc);
+          if (z >= zs) store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc[0]);
+          shift_queue<T, NZ, M, VX>(acc);
+        } else {
+          static_for<0, NZ>([&](auto ic) {
+            constexpr int UR = decltype(ic)::value;
+            if (ur == UR) {
+              zero_acc<T, VX, M>(acc[UR]);
+              run_scatter<S, VX, M, UR>(pl, acc);
+              if (z >= zs) store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc[(UR + 1) % NZ]);
+            }
+          });
+        }
       }
       __syncthreads();
     }
@@ -1009,16 +1053,19 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     T acc[NZ][MI][VX];
 #pragma unroll
     for (int q = 0; q < NZ; ++q) zero_acc<T, VX, MI>(acc[q]);
+    // NZ unrolled plane bodies (compile-time queue rotation), or one body and
+    // a register shift of the queue for large op tables (S::RTSHIFT)
+    constexpr int UNR = S::RTSHIFT ? 1 : NZ;
 #pragma unroll 1
-    for (int jb = 0; jb < nin; jb += NZ) {
-      static_for<0, NZ>([&](auto ic) {
-        constexpr int U = decltype(ic)::value;
-        const int j = jb + U;
+    for (int jb = 0; jb < nin; jb += UNR) {
+      static_for<0, UNR>([&](auto ic) {
+        constexpr int U = S::RTSHIFT ? NZ - 1 : decltype(ic)::value;
+        const int j = jb + decltype(ic)::value;
         if (j >= nin) return;
         const int si = j % DIN;
         const T* src = s == 1 ? ring0 + si * C::PLANE : mid + (2 * (s - 2) + si) * C::PLANE;
         mbar_wait_sleep(&fin[si], (unsigned)((j / DIN) & 1));
-        zero_acc<T, VX, MI>(acc[U]);                     // a new output plane starts
+        if constexpr (!S::RTSHIFT) zero_acc<T, VX, MI>(acc[U]);   // a new output plane starts
         if (act) {
           SmemPlane<T, VX, C::LX> pl{src + lb};
           run_scatter_ops<S, typename S::Mid, VX, MI, U>(pl, acc);
@@ -1056,6 +1103,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
           }
         }
         mbar_arrive(&full_s(s)[so]);                     // stage-s plane written
+        if constexpr (S::RTSHIFT) shift_queue<T, NZ, MI, VX>(acc);
       });
     }
   });
@@ -1076,15 +1124,16 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     T acc[NZ][M][VX];
 #pragma unroll
     for (int u = 0; u < NZ; ++u) zero_acc<T, VX, M>(acc[u]);
+    constexpr int UNR = S::RTSHIFT ? 1 : NZ;
 #pragma unroll 1
-    for (int jb = 0; jb < nin; jb += NZ) {
-      static_for<0, NZ>([&](auto ic) {
-        constexpr int U = decltype(ic)::value;
-        const int j = jb + U;
+    for (int jb = 0; jb < nin; jb += UNR) {
+      static_for<0, UNR>([&](auto ic) {
+        constexpr int U = S::RTSHIFT ? NZ - 1 : decltype(ic)::value;
+        const int j = jb + decltype(ic)::value;
         if (j >= nin) return;
         const int si = j & 1;
         mbar_wait_sleep(&fin[si], (unsigned)((j >> 1) & 1));
-        zero_acc<T, VX, M>(acc[U]);
+        if constexpr (!S::RTSHIFT) zero_acc<T, VX, M>(acc[U]);
         if (act) {
           SmemPlane<T, VX, C::LX> pl{mid + (2 * (TT - 2) + si) * C::PLANE + row0 * C::LX + col0};
           run_scatter<S, VX, M, U>(pl, acc);
@@ -1092,6 +1141,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         mbar_arrive(&ein[si]);
         const int z = pin0 + j - TT * S::ZHI;
         if (act && z >= zs) ts.store(z, acc[(U + 1) % NZ]);
+        if constexpr (S::RTSHIFT) shift_queue<T, NZ, M, VX>(acc);
       });
     }
   }

@@ -320,6 +320,15 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   o << "  static __device__ __forceinline__ constexpr int idx(int z, int y, int x) { return g_idx[z][y][x]; }\n";
   o << "  static __device__ __forceinline__ constexpr T coef(int i) { return g_coef[i]; }\n";
   o << "  static constexpr int NOPS = " << ops.size() << ";\n";
+  // retiming queue rotation: NZ unrolled plane bodies while they stay small,
+  // register shifts beyond. Measured (B200, 512^3 / 768^3): the unrolled form
+  // is instruction-cache bound on a 293-point order-4 stencil ('no_instructions'
+  // the top stall; 27 -> 51 GStencil/s with shifts) and on an order-3 one
+  // (55 -> 84); it wins on the 25-point star (567 vs 493, ops*NZ ~ 2100) and
+  // the heat stencil. Crossover between ~2100 and ~2500 table entries x NZ.
+  int rtshift = (long)ops.size() * NZ > 2300 ? 1 : 0;
+  if (const char* e = getenv("STENCIL_RT_SHIFT")) rtshift = atoi(e);   // dev override
+  o << "  static constexpr int RTSHIFT = " << rtshift << ";\n";
   o << "  static __device__ __forceinline__ constexpr unsigned op(int i) { return g_ops[i]; }\n";
   o << "};\n}  // namespace gen\n";
   o << "// variant: " << v.name_expr("gen::S") << "\n";
@@ -339,9 +348,15 @@ int compile_variant(const Pattern& pat, int dtype, const Variant& v, std::string
       return STENCIL_OK;
     }
   }
-  const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "-default-device",
-                        "--extra-device-vectorization"};
-  const int nopt = sizeof(opts) / sizeof(opts[0]);
+  std::vector<const char*> optv = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "-default-device",
+                                   "--extra-device-vectorization"};
+  static thread_local std::string maxreg_opt;
+  if (const char* e = getenv("STENCIL_MAXRREG")) {   // dev override (register cap experiments)
+    maxreg_opt = std::string("--maxrregcount=") + e;
+    optv.push_back(maxreg_opt.c_str());
+  }
+  const char* const* opts = optv.data();
+  const int nopt = (int)optv.size();
   int nv_major = 0, nv_minor = 0;
   nvrtcVersion(&nv_major, &nv_minor);
   std::string key_str = src + "|" + kKernelsSrc + "|";

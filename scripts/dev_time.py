@@ -11,9 +11,10 @@ ap.add_argument("--ocs", default="all")
 ap.add_argument("--steps", type=int, default=10)
 ap.add_argument("--reps", type=int, default=3)
 ap.add_argument("--params", default="{}")
+ap.add_argument("--stencil", default="")
 a = ap.parse_args()
 C = si.CONFIGS[a.cfg]
-acc, c = si.config_stencil(C["stencil"] if C["stencil"] != "random3d" else "random3d:2:1")
+acc, c = si.config_stencil(a.stencil or (C["stencil"] if C["stencil"] != "random3d" else "random3d:2:1"))
 dims, dtype = C["dims"], C["dtype"]
 tdt = torch.float64 if dtype == "f64" else torch.float32
 x = torch.empty(dims, dtype=tdt, device="cuda"); sm.fill_field(x, C["seed"])
