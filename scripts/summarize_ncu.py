@@ -43,32 +43,44 @@ def full_report(rep, out_json):
     return res
 
 
-def launches(csv_path, out_md, title):
+def _table(f, seq):
+    agg = collections.OrderedDict()
+    tot = 0.0
+    for name, ns in seq:
+        a = agg.setdefault(name, [0, 0.0])
+        a[0] += 1
+        a[1] += ns
+        tot += ns
+    f.write(f'Launches: {len(seq)}, total kernel time {tot / 1e6:.3f} ms\n\n'
+            '| kernel | launches | total ms | mean us | share |\n|---|---|---|---|---|\n')
+    for k, (n, ns) in sorted(agg.items(), key=lambda kv: -kv[1][1]):
+        f.write(f'| `{k[:110]}` | {n} | {ns / 1e6:.3f} | {ns / n / 1e3:.1f} | {ns / tot:.3f} |\n')
+
+
+def launches(csv_path, out_md, title, tail=0):
+    """Whole launch list; with tail=N also the last N launches (the bench's
+    timed region: its JSON line reports gpu_launches = N)."""
     rows = list(csv.reader(open(csv_path)))
     hi = [i for i, r in enumerate(rows) if r and r[0] == 'ID'][0]
     h = rows[hi]
-    agg = collections.OrderedDict()
-    tot = 0.0
+    seq = []
     for r in rows[hi + 1:]:
         d = dict(zip(h, r))
         if d.get('Metric Name') != 'gpu__time_duration.sum':
             continue
-        ns = float(d['Metric Value'].replace(',', ''))
-        a = agg.setdefault(d['Kernel Name'], [0, 0.0])
-        a[0] += 1
-        a[1] += ns
-        tot += ns
+        seq.append((d['Kernel Name'], float(d['Metric Value'].replace(',', ''))))
     with open(out_md, 'w') as f:
         f.write(f'# {title}\n\nncu launch list (`--metrics gpu__time_duration.sum --clock-control none`), '
                 'cold-cache and serialised: compare shares, not absolutes.\n\n')
-        f.write(f'Total launches: {sum(a[0] for a in agg.values())}, total kernel time {tot / 1e6:.3f} ms\n\n'
-                '| kernel | launches | total ms | mean us | share |\n|---|---|---|---|---|\n')
-        for k, (n, ns) in sorted(agg.items(), key=lambda kv: -kv[1][1]):
-            f.write(f'| `{k[:110]}` | {n} | {ns / 1e6:.3f} | {ns / n / 1e3:.1f} | {ns / tot:.3f} |\n')
+        if tail:
+            f.write(f'## Timed region (the last {tail} launches = the JSON line\'s gpu_launches)\n\n')
+            _table(f, seq[-tail:])
+            f.write('\n## Whole run (label pass over all OCs + warm-up + timed region)\n\n')
+        _table(f, seq)
 
 
 if __name__ == '__main__':
     if sys.argv[1] == 'full':
         full_report(sys.argv[2], sys.argv[3])
     else:
-        launches(sys.argv[2], sys.argv[3], sys.argv[4])
+        launches(sys.argv[2], sys.argv[3], sys.argv[4], int(sys.argv[5]) if len(sys.argv) > 5 else 0)

@@ -68,6 +68,12 @@ CASES = [
     ("random3d:2:5", (27, 33, 44), "f64", 2),
     ("random3d:3:1", (24, 26, 36), "f32", 2),
     ("random3d:4:3", (25, 23, 40), "f64", 1),
+    # NEXT-2: random 2-D stencils (Algorithm 1, d = 2) under all 30 OCs; the
+    # streaming OCs stream along y (C-13)
+    ("random2d:1:0", (70, 90), "f64", 4),
+    ("random2d:2:4", (45, 130), "f64", 3),
+    ("random2d:3:8", (61, 77), "f32", 2),
+    ("random2d:4:12", (50, 68), "f64", 2),
 ]
 
 
@@ -189,14 +195,17 @@ def test_oc_sweep_label(gpu):
     assert _relerr(y.cpu().numpy(), ref) <= 1e-12
 
 
-@pytest.mark.parametrize("cfg,ocs", [("C2", ["ST_RT_PR", "ST_PR", "base"]), ("C3", ["ST_RT_PR", "ST_BM_PR"]),
-                                     ("C4", ["ST_RT_PR", "TB"])])
-def test_full_size_sampled(gpu, cfg, ocs):
-    """BASELINE sizes, the bench's launch configuration, sampled points vs
-    the oracle on their dependency cones."""
+@pytest.mark.parametrize("cfg,ocs,stencil", [
+    ("C2", ["ST_RT_PR", "ST_PR", "base", "ST_TB_BM_RT_PR"], None), ("C3", ["ST_RT_PR", "ST_BM_RT_PR"], None),
+    ("C4", ["ST_RT_PR", "TB"], None), ("C5", ["ST_BM_RT_PR"], "random3d:4:12"),
+    ("C5", ["ST_TB_BM_RT_PR"], "random3d:1:0"), ("N2", ["TB_BM", "ST_BM_RT_PR"], "random2d:3:8")])
+def test_full_size_sampled(gpu, cfg, ocs, stencil):
+    """BASELINE sizes, the bench's launch configuration (default settings of
+    the OCs the bench labels), sampled points vs the oracle on their
+    dependency cones."""
     torch = _torch()
     C = si.CONFIGS[cfg]
-    acc, c = si.config_stencil(C["stencil"])
+    acc, c = si.config_stencil(stencil or C["stencil"])
     dims, dtype, steps = C["dims"], C["dtype"], C["steps"]
     tdt = torch.float64 if dtype == "f64" else torch.float32
     x = torch.empty(dims, dtype=tdt, device="cuda")
@@ -204,8 +213,10 @@ def test_full_size_sampled(gpu, cfg, ocs):
     y = torch.empty_like(x)
     rng = np.random.default_rng(0)
     pts = np.stack([rng.integers(0, n, size=24) for n in dims], axis=1)
-    pts = np.concatenate([pts, [[0, 0, 0], [4, 4, 4], [dims[0] - 5, dims[1] - 1, dims[2] - 6],
-                                [dims[0] // 2, 4, dims[2] - 5]]])
+    nd = len(dims)
+    edge = [[0] * nd, [4] * nd, [d - 5 for d in dims[:-1]] + [dims[-1] - 6],       # frame, near-frame
+            [dims[0] // 2] + [4] * (nd - 2) + [dims[-1] - 5], [d - 1 for d in dims]]
+    pts = np.concatenate([pts, np.array(edge, dtype=pts.dtype)])
     ref = oracle.sweep_points(pts, dims, C["seed"], "uniform12", acc, c, steps, dtype)
     for name in ocs:
         p = sm.Plan(dims, acc, c, dtype, sm.oc_from_name(name))
