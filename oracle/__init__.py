@@ -25,9 +25,15 @@ Functions and the passages they follow:
   hand-built vectors.
 * :func:`features` -- Table II features. Pinned by star / box
   closed forms (nnz = 2dr+1, (2r+1)^d; ring sizes (2k+1)^d - (2k-1)^d).
+* :mod:`oracle.oc_groups` -- the OC analysis between labelling and
+  classification: Fig. 1 gap, Fig. 2 wins,
+  Fig. 3 pairwise PCC and the PCC merge into 5 classes (P:L107,
+  P:L186). Pinned by tests/test_oc_groups_pins.py (scipy pearsonr,
+  scipy single-linkage clustering, hand-built matrices).
 """
+from . import oc_groups
 from .oracle import (OC_BITS, best_oc, build_oracle, features, max_threads, oc_name,
                      sweep, sweep_points, valid_ocs)
 
-__all__ = ["OC_BITS", "best_oc", "build_oracle", "features", "max_threads", "oc_name",
+__all__ = ["oc_groups", "OC_BITS", "best_oc", "build_oracle", "features", "max_threads", "oc_name",
            "sweep", "sweep_points", "valid_ocs"]
