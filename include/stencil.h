@@ -244,6 +244,32 @@ typedef struct {
 int stencil_sweep_rows(stencil_plan_t plan, stencil_sweep_row_t *rows, int max_rows, int *nrows);
 
 /* ---------------------------------------------------------------------------
+ * OC analysis over a stencil dataset (§III-A..C, §IV-D, §V-A.2;
+ * SURVEY NEXT-4; host only, no CUDA call)
+ * ------------------------------------------------------------------------- */
+
+/* times: [n_stencils][n_oc] row-major host array of per-OC shortest times
+ * (ms; a value that is not finite and > 0 = the OC did not run on that
+ * stencil). 1 <= n_oc <= 64, n_classes >= 1. Every output is optional
+ * (NULL = not wanted), host memory owned by the caller:
+ *   gap[n_stencils]   worst / best time per stencil (Fig. 1); NaN if no OC ran;
+ *   wins[n_oc]        stencils each OC is best for (Fig. 2; ties -> smaller column);
+ *   pcc[n_oc*n_oc]    Pearson correlation between OC columns of the per-stencil
+ *                     performance t_best/t, over the stencils where both ran
+ *                     (Fig. 3); < 3 common stencils or zero variance -> 0;
+ *   group[n_oc]       class of each OC after merging pairs by |PCC| descending
+ *                     (ties -> smaller (a,b)) until n_classes groups remain
+ *                     ("reduce the number of predicted
+ *                     OCs to 5"); groups numbered by their smallest member;
+ *   rep[n_classes]    the member with the most wins ("the OC that obtains
+ *                     the best performance under more cases"; ties -> smaller
+ *                     column); -1 for unused classes when n_oc < n_classes;
+ *   labels[n_stencils] class of each stencil = group of its best OC, -1 if none ran.
+ * Errors: E_INVAL on bad sizes or a null `times` with n_stencils > 0. */
+int stencil_oc_analysis(int n_stencils, int n_oc, const double *times, int n_classes, double *gap,
+                        int32_t *wins, double *pcc, int32_t *group, int32_t *rep, int32_t *labels);
+
+/* ---------------------------------------------------------------------------
  * Synthetic inputs (the counter-based generator of DESIGN.md, reading C-3)
  * ------------------------------------------------------------------------- */
 

@@ -7,10 +7,10 @@ is its thin ctypes binding.
 """
 from .binding import (F32, F64, NUM_OC, OC_BM, OC_CM, OC_PR, OC_RT, OC_ST, OC_TB, Plan, StencilError,
                       embed_tensor, exported_symbols, features, fill_field, gstencil_per_s, launch_count, lib,
-                      link_loopback, nccl_unique_id, oc_from_name, oc_list, oc_name, oc_valid, run_group,
+                      link_loopback, nccl_unique_id, oc_analysis, oc_from_name, oc_list, oc_name, oc_valid, run_group,
                       sample_params, slab_halo, slab_range)
 
 __all__ = ["F32", "F64", "NUM_OC", "OC_BM", "OC_CM", "OC_PR", "OC_RT", "OC_ST", "OC_TB", "Plan", "StencilError",
            "embed_tensor", "exported_symbols", "features", "fill_field", "gstencil_per_s", "launch_count", "lib",
-           "link_loopback", "nccl_unique_id", "oc_from_name", "oc_list", "oc_name", "oc_valid", "run_group",
+           "link_loopback", "nccl_unique_id", "oc_analysis", "oc_from_name", "oc_list", "oc_name", "oc_valid", "run_group",
            "sample_params", "slab_halo", "slab_range"]

@@ -78,6 +78,9 @@ _SIGS = {
     "stencil_embed_tensor": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p]),
     "stencil_sweep_rows": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(SweepRow), ctypes.c_int,
                                           ctypes.POINTER(ctypes.c_int)]),
+    "stencil_oc_analysis": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
+                                           ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                           ctypes.c_void_p, ctypes.c_void_p]),
     "stencil_plan_create": (ctypes.c_int, [ctypes.POINTER(ctypes.c_void_p), ctypes.c_int,
                                            ctypes.POINTER(ctypes.c_int64), ctypes.c_int, ctypes.c_void_p,
                                            ctypes.c_void_p, ctypes.c_int, ctypes.c_uint32,
@@ -221,6 +224,26 @@ def embed_tensor(access: np.ndarray) -> np.ndarray:
     out = np.zeros((9,) * acc.ndim, dtype=np.uint8)
     _check(lib().stencil_embed_tensor(acc.ndim, (acc.shape[0] - 1) // 2, acc.ctypes.data, out.ctypes.data))
     return out
+
+
+def oc_analysis(times, n_classes: int = 5) -> Dict[str, object]:
+    """OC analysis of a (stencil x OC) matrix of per-OC shortest times:
+    Fig. 1 gap, Fig. 2 wins, Fig. 3 PCC matrix, the PCC merge into n_classes
+    groups with their representatives, and each stencil's class (stencil_oc_analysis)."""
+    t = np.ascontiguousarray(np.asarray(times, dtype=np.float64))
+    if t.ndim != 2:
+        raise ValueError("times must be [n_stencils][n_oc]")
+    ns, k = t.shape
+    gap = np.zeros(ns, dtype=np.float64)
+    wins = np.zeros(k, dtype=np.int32)
+    pcc = np.zeros((k, k), dtype=np.float64)
+    group = np.zeros(k, dtype=np.int32)
+    rep = np.zeros(max(n_classes, 1), dtype=np.int32)
+    labels = np.zeros(ns, dtype=np.int32)
+    _check(lib().stencil_oc_analysis(ns, k, t.ctypes.data, n_classes, gap.ctypes.data, wins.ctypes.data,
+                                     pcc.ctypes.data, group.ctypes.data, rep.ctypes.data, labels.ctypes.data))
+    return {"gap": gap, "wins": wins, "pcc": pcc, "group": group.tolist(),
+            "representative": [int(r) for r in rep if r >= 0], "labels": labels.tolist()}
 
 
 def slab_halo(ghost: int, n: int, zlo_g: int, zhi_g: int, rank: int, nranks: int) -> Dict[str, Tuple[int, int]]:

@@ -67,3 +67,25 @@ def append_rows(path: str, rows: Iterable[dict]) -> None:
             f.write(json.dumps(r) + "\n")
         f.flush()
         os.fsync(f.fileno())
+
+
+def load_matrix(path: str, ndim: Optional[int] = None):
+    """(stencil ids, OC names, [n_stencils][30] per-OC shortest times in ms, +inf =
+    infeasible) from the label lines of a dataset file -- the input of the OC
+    analysis ("the shortest execution time of each OC under different
+    parameter settings is used for OC selection")."""
+    from .binding import oc_list
+    names = [oc_name(o) for o in oc_list()]
+    ids, rows = [], []
+    with open(path) as f:
+        for line in f:
+            try:
+                d = json.loads(line)
+            except json.JSONDecodeError:
+                continue
+            if d.get("kind") != "label" or (ndim is not None and d.get("ndim") != ndim):
+                continue
+            t = d["oc_times_ms"]
+            ids.append(d["stencil_id"])
+            rows.append([math.inf if t.get(n) is None else float(t[n]) for n in names])
+    return ids, names, np.array(rows, dtype=np.float64).reshape(len(rows), len(names))
