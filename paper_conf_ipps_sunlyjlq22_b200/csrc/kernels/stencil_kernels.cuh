@@ -16,6 +16,7 @@
 //   static __device__ constexpr T coef(int i);
 //   static constexpr int NOPS; static __device__ constexpr unsigned op(int i);
 //       the variant's op table (see run_gather / run_scatter).
+//   static constexpr int MIDR;  slots of each intermediate-stage ring of k_stream_tb_rt.
 //   static constexpr int RTSHIFT;  1: retiming queues rotate by register
 //       shifts (one plane body) instead of NZ unrolled bodies (large tables).
 //
@@ -156,6 +157,15 @@ __device__ __forceinline__ void stg_vec(T* p, const T (&w)[VX]) {
 __device__ __forceinline__ double fma_t(double a, double b, double c) { return __fma_rn(a, b, c); }
 __device__ __forceinline__ float fma_t(float a, float b, float c) { return __fmaf_rn(a, b, c); }
 
+// packed op (fp32 only, emitted by the generator): a0 += c*w0, a1 += c*w1 as one
+// FFMA2 -- per lane an ordinary RN fma, so results are bitwise those of fma_t
+__device__ __forceinline__ void fma2_t(float c, float w0, float w1, float& a0, float& a1) {
+  const float2 r = __ffma2_rn(make_float2(w0, w1), make_float2(c, c), make_float2(a0, a1));
+  a0 = r.x;
+  a1 = r.y;
+}
+__device__ __forceinline__ void fma2_t(double, double, double, double&, double&) {}   // never emitted
+
 // ---------------------------------------------------------------------------
 // compile-time pattern predicates (fold to constants after unrolling)
 // ---------------------------------------------------------------------------
@@ -210,7 +220,8 @@ struct GlobalPlane {                  // global memory through the read-only pat
 //                     vector kv = ((op >> 12) & 15) - 8  (columns [kv*VX, kv*VX+VX))
 //   FMA  (bit31 = 1): coefficient id = op & 1023, element e = (op >> 10) & 3,
 //                     output column v = (op >> 12) & 3, output row m = (op >> 14) & 7,
-//                     slice zi = (op >> 17) & 15
+//                     slice zi = (op >> 17) & 15; bit 30 (fp32 only): packed pair,
+//                     columns v, v+1 from elements e, e+1 (one FFMA2)
 // The generator emits each value once per window and, per accumulator, the
 // FMAs in lexicographic (dz, dy, dx) order.
 // run_gather:  out plane z reads plane z + zi - ZLO through pl[zi].
@@ -229,6 +240,9 @@ __device__ __forceinline__ void run_gather_ops(const L (&pl)[S::NZ], typename S:
     const unsigned op = O::op(i);
     if (!(op >> 31)) {
       pl[op & 15].get(int((op >> 4) & 255) - 128, int((op >> 12) & 15) - 8, w);
+    } else if (op & 0x40000000u) {
+      T* a = &acc[(op >> 14) & 7][(op >> 12) & 3];
+      fma2_t(S::coef(op & 1023), w[(op >> 10) & 3], w[((op >> 10) & 3) + 1], a[0], a[1]);
     } else {
       T& a = acc[(op >> 14) & 7][(op >> 12) & 3];
       a = fma_t(S::coef(op & 1023), w[(op >> 10) & 3], a);
@@ -251,6 +265,10 @@ __device__ __forceinline__ void run_scatter_ops(const L& pl, typename S::T (&acc
     const unsigned op = O::op(i);
     if (!(op >> 31)) {
       pl.get(int((op >> 4) & 255) - 128, int((op >> 12) & 15) - 8, w);
+    } else if (op & 0x40000000u) {
+      const int zi = (op >> 17) & 15;
+      T* a = &acc[(U + NZ - zi) % NZ][(op >> 14) & 7][(op >> 12) & 3];
+      fma2_t(S::coef(op & 1023), w[(op >> 10) & 3], w[((op >> 10) & 3) + 1], a[0], a[1]);
     } else {
       const int zi = (op >> 17) & 15;
       T& a = acc[(U + NZ - zi) % NZ][(op >> 14) & 7][(op >> 12) & 3];
@@ -892,12 +910,15 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
 // step is about that of one ST sweep while HBM traffic is divided by TT.
 //
 // Warp-specialised pipeline (no CTA-wide barrier in the loop):
-//   warp 0, lane 0  producer: TMA loads of input planes into an NS-slot ring
-//                   (NS = planes in flight: PR; NS = 1 is "no prefetching");
+//   warp 0, lane 0  producer: TMA loads of input planes into an NR-slot ring
+//                   (NS = planes in flight: PR; NS = 1 is "no prefetching";
+//                   NR = NS + ZHI because stage 1 keeps input plane j - ZHI
+//                   until iteration j: it is the frame source of the stage-1
+//                   plane completed then);
 //   group s=1..TT-1 one VX x MI register tile per thread over region R_s
 //                   (the output tile expanded by (TT-s)*extent), op table
-//                   S::Mid in scatter form; writes stage-s planes into a
-//                   2-slot ring;
+//                   S::Mid in scatter form; writes stage-s planes into an
+//                   MR-slot ring (S::MIDR);
 //   group TT        the M x VX (BM/CM) output tile of k_stream, scatter form,
 //                   stores to HBM.
 // Hand-offs are mbarriers: full[slot] (count = producer threads; TMA: tx
@@ -908,8 +929,8 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
 // Tile values outside R_s are computed from don't-care inputs and never feed
 // a valid output, so they are stored unmasked (inside the plane buffer).
 // Frame points (outside the update box) keep their value at every fused step
-// and read it from the launch's input grid (the frame never changes,
-// DESIGN.md C-1). Canonical order (C-4): partial sums receive slices in
+// (the frame never changes, C-1): stage 1 takes it from the input
+// plane still held in the ring, later stages from the launch's input grid. Canonical order (C-4): partial sums receive slices in
 // ascending dz and, in each slice, FMAs in (dy,dx) order -- bitwise equal to
 // every other OC.
 // ===========================================================================
@@ -945,8 +966,10 @@ struct StreamTbRtCfg {
   static constexpr int MI = S::MI;
   static constexpr int PADF = 128 / (int)sizeof(T);
   static constexpr int PADB = ((MI * LX + ALN) * (int)sizeof(T) + 127) / 128 * 128 / (int)sizeof(T);
-  static constexpr int ELEMS = PADF + (NS + 2 * (TT - 1)) * PLANE + PADB;
-  static constexpr int NBAR = 2 * NS + 4 * (TT - 1);
+  static constexpr int NR = NS + S::ZHI;                     // input ring slots
+  static constexpr int MR = S::MIDR;                         // slots of each stage ring
+  static constexpr int ELEMS = PADF + (NR + MR * (TT - 1)) * PLANE + PADB;
+  static constexpr int NBAR = 2 * NR + 2 * MR * (TT - 1);
   static constexpr int SMEM = ELEMS * (int)sizeof(T) + 8 * NBAR + 128;
   static constexpr int FT = (BX / VX) * BY;                 // last-stage tiles
   static constexpr int WF = (FT + 31) / 32;
@@ -962,17 +985,18 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
   typedef StreamTbRtCfg<S, BX, BY, VX, M, CM, NS, TT> C;
   constexpr int NZ = S::NZ;
   constexpr int MI = C::MI;
+  constexpr int NR = C::NR, MR = C::MR;
   static_assert(TT >= 2, "k_stream_tb_rt needs TT >= 2");
   extern __shared__ __align__(128) unsigned char smem_raw[];
   T* sbase = reinterpret_cast<T*>(smem_raw);
   T* ring0 = sbase + C::PADF;
-  T* mid = ring0 + NS * C::PLANE;                      // stage s slot b: mid + (2*(s-1)+b)*PLANE
+  T* mid = ring0 + NR * C::PLANE;                      // stage s slot b: mid + (MR*(s-1)+b)*PLANE
   unsigned long long* bars = reinterpret_cast<unsigned long long*>(smem_raw + C::ELEMS * sizeof(T));
-  // bars: full_in[NS], empty_in[NS], then per stage s=1..TT-1: full_s[2], empty_s[2]
+  // bars: full_in[NR], empty_in[NR], then per stage s=1..TT-1: full_s[MR], empty_s[MR]
   unsigned long long* full_in = bars;
-  unsigned long long* empty_in = bars + NS;
-  auto full_s = [&](int s) { return bars + 2 * NS + 4 * (s - 1); };
-  auto empty_s = [&](int s) { return bars + 2 * NS + 4 * (s - 1) + 2; };
+  unsigned long long* empty_in = bars + NR;
+  auto full_s = [&](int s) { return bars + 2 * NR + 2 * MR * (s - 1); };
+  auto empty_s = [&](int s) { return bars + 2 * NR + 2 * MR * (s - 1) + MR; };
 
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
@@ -989,14 +1013,14 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
   for (int i = tid; i < C::ELEMS; i += C::THREADS) sbase[i] = T(0);
   if (tid == 0) {
     tma_prefetch_desc(&tmap);
-    for (int q = 0; q < NS; ++q) {
+    for (int q = 0; q < NR; ++q) {
       mbar_init(&full_in[q], 1);
       mbar_init(&empty_in[q], 32 * TbRtStage<S, BX, BY, VX, M, TT, MI, 1>::W);
     }
     static_for<1, TT>([&](auto sc) {
       constexpr int s = decltype(sc)::value;
       constexpr int WN = s + 1 < TT ? TbRtStage<S, BX, BY, VX, M, TT, MI, s + 1>::W : C::WF;
-      for (int b = 0; b < 2; ++b) {
+      for (int b = 0; b < MR; ++b) {
         mbar_init(&full_s(s)[b], 32 * TbRtStage<S, BX, BY, VX, M, TT, MI, s>::W);
         mbar_init(&empty_s(s)[b], 32 * WN);
       }
@@ -1011,8 +1035,8 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     if (tid == 0) {
 #pragma unroll 1
       for (int j = 0; j < nin; ++j) {
-        const int slot = j % NS;
-        if (j >= NS) mbar_wait_sleep(&empty_in[slot], (unsigned)((j / NS - 1) & 1));
+        const int slot = j % NR;
+        if (j >= NR) mbar_wait_sleep(&empty_in[slot], (unsigned)((j / NR - 1) & 1));
         mbar_expect_tx(&full_in[slot], C::LX * C::LY * (unsigned)sizeof(T));
         tma_load_3d(ring0 + slot * C::PLANE, &tmap, &full_in[slot], X0, Y0, pin0 + j);
       }
@@ -1049,7 +1073,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     const bool fast = act && xfast && allup;
     unsigned long long* fin = s == 1 ? full_in : full_s(s - 1);
     unsigned long long* ein = s == 1 ? empty_in : empty_s(s - 1);
-    constexpr int DIN = s == 1 ? NS : 2;
+    constexpr int DIN = s == 1 ? NR : MR;
     T acc[NZ][MI][VX];
 #pragma unroll
     for (int q = 0; q < NZ; ++q) zero_acc<T, VX, MI>(acc[q]);
@@ -1063,18 +1087,20 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         const int j = jb + decltype(ic)::value;
         if (j >= nin) return;
         const int si = j % DIN;
-        const T* src = s == 1 ? ring0 + si * C::PLANE : mid + (2 * (s - 2) + si) * C::PLANE;
+        const T* src = s == 1 ? ring0 + si * C::PLANE : mid + (MR * (s - 2) + si) * C::PLANE;
         mbar_wait_sleep(&fin[si], (unsigned)((j / DIN) & 1));
         if constexpr (!S::RTSHIFT) zero_acc<T, VX, MI>(acc[U]);   // a new output plane starts
         if (act) {
           SmemPlane<T, VX, C::LX> pl{src + lb};
           run_scatter_ops<S, typename S::Mid, VX, MI, U>(pl, acc);
         }
-        mbar_arrive(&ein[si]);                           // input slot read
-        const int so = j & 1;
-        T* dst = mid + (2 * (s - 1) + so) * C::PLANE;
-        if (j >= 2) mbar_wait_sleep(&empty_s(s)[so], (unsigned)((j / 2 - 1) & 1));
+        if (s > 1) mbar_arrive(&ein[si]);                // input slot read (stage 1: below)
+        const int so = j % MR;
+        T* dst = mid + (MR * (s - 1) + so) * C::PLANE;
+        if (j >= MR) mbar_wait_sleep(&empty_s(s)[so], (unsigned)((j / MR - 1) & 1));
         const int zo = pin0 + j - s * S::ZHI;            // plane completed now
+        // stage 1: input plane zo (= index j - ZHI) is still in the ring
+        const T* fr = ring0 + ((j - S::ZHI + NR) % NR) * C::PLANE + lb;
         const bool zin = zo >= 0 && zo < g.nz;
         const bool zupd = zo >= g.uz0 && zo < g.uz1;
         const T(&res)[MI][VX] = acc[(U + 1) % NZ];
@@ -1097,11 +1123,12 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
                 const int gx = gx0 + v;
                 if (gx < 0 || gx >= g.nx || gx - X0 >= C::LX) continue;
                 const bool upd = rowupd && gx >= g.ux0 && gx < g.ux1;
-                d[v] = upd ? res[m][v] : __ldg(frame + gx);
+                d[v] = upd ? res[m][v] : (s == 1 ? fr[m * C::LX + v] : __ldg(frame + gx));
               }
             }
           }
         }
+        if (s == 1 && j >= S::ZHI) mbar_arrive(&ein[(j - S::ZHI) % NR]);   // frame source released
         mbar_arrive(&full_s(s)[so]);                     // stage-s plane written
         if constexpr (S::RTSHIFT) shift_queue<T, NZ, MI, VX>(acc);
       });
@@ -1131,11 +1158,11 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         constexpr int U = S::RTSHIFT ? NZ - 1 : decltype(ic)::value;
         const int j = jb + decltype(ic)::value;
         if (j >= nin) return;
-        const int si = j & 1;
-        mbar_wait_sleep(&fin[si], (unsigned)((j >> 1) & 1));
+        const int si = j % MR;
+        mbar_wait_sleep(&fin[si], (unsigned)((j / MR) & 1));
         if constexpr (!S::RTSHIFT) zero_acc<T, VX, M>(acc[U]);
         if (act) {
-          SmemPlane<T, VX, C::LX> pl{mid + (2 * (TT - 2) + si) * C::PLANE + row0 * C::LX + col0};
+          SmemPlane<T, VX, C::LX> pl{mid + (MR * (TT - 2) + si) * C::PLANE + row0 * C::LX + col0};
           run_scatter<S, VX, M, U>(pl, acc);
         }
         mbar_arrive(&ein[si]);

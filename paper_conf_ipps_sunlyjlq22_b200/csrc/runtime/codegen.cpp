@@ -140,6 +140,12 @@ int Variant::mid_rows(const Pattern& p, int elem) const {
   return 2;
 }
 
+// Slots of each intermediate-stage ring of k_stream_tb_rt (S::MIDR).
+int Variant::mid_slots() const {
+  if (const char* e = getenv("STENCIL_MIDR")) return std::max(2, atoi(e));   // dev override
+  return 2;
+}
+
 // Mirrors StreamTbRtCfg::THREADS of stencil_kernels.cuh: one producer warp,
 // ceil(NT_s / 32) warps per intermediate stage s, ceil(tiles / 32) last-stage warps.
 int Variant::tbrt_threads(const Pattern& p, int elem) const {
@@ -184,7 +190,8 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     const int plane = roundup(lx * ly * elem, 128) / elem;
     const int padf = 128 / elem;
     const int padb = roundup((mid_rows(p, elem) * lx + aln) * elem, 128) / elem;
-    return (padf + (ns + 2 * (tt - 1)) * plane + padb) * elem + 8 * (2 * ns + 4 * (tt - 1)) + 128;
+    const int nr = ns + p.zhi, mr = mid_slots();
+    return (padf + (nr + mr * (tt - 1)) * plane + padb) * elem + 8 * (2 * nr + 2 * mr * (tt - 1)) + 128;
   }
   if (family == FAM_STREAM_TB) {   // mirrors StreamTbCfg
     const int xoff = roundup(tt * p.xlo, aln);
@@ -203,7 +210,13 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
 // Op table of a variant (format documented at run_gather in stencil_kernels.cuh).
 // Loops are ordered so that every accumulator receives its FMAs in
 // lexicographic (dz, dy, dx) order -- the canonical chain of every OC.
-static std::vector<uint32_t> encode_ops(const Pattern& pat, const Variant& v) {
+// fp32 (`pair`): two FMAs that share a coefficient and feed adjacent output
+// columns (v, v+1) from adjacent window elements (e, e+1), v and e even, become
+// ONE packed op (bit 30) that the kernels issue as an FFMA2 (sm_100's packed
+// fp32 FMA: two independent RN fmas, so every chain stays bitwise the same).
+// The window's FMAs are emitted offset-major (dx ascending, then column), which
+// keeps each accumulator's chain lexicographic and puts pair partners side by side.
+static std::vector<uint32_t> encode_ops(const Pattern& pat, const Variant& v, bool pair) {
   const int NZ = pat.zlo + pat.zhi + 1, NY = pat.ylo + pat.yhi + 1, NX = pat.xlo + pat.xhi + 1;
   std::vector<int> idx((size_t)NZ * NY * NX, -1);
   for (int i = 0; i < pat.nnz; ++i)
@@ -228,13 +241,23 @@ static std::vector<uint32_t> encode_ops(const Pattern& pat, const Variant& v) {
     // FMAs fed by window (row j_rel, vector kv); jbase = j_rel - (row of output m_lo's dy = 0)
     f.clear();
     for (int zi = zi_lo; zi < zi_hi; ++zi)
-      for (int m = m_lo; m < m_hi; ++m)
-        for (int vv = 0; vv < VX; ++vv)
-          for (int e = 0; e < VX; ++e) {
-            const int dyi = (v.cm ? jbase : jbase - m) + pat.ylo;
-            const int id = cidx(zi, dyi, kv * VX + e - vv + pat.xlo);
-            if (id >= 0) f.push_back(fma(id, e, vv, m, zi));
+      for (int m = m_lo; m < m_hi; ++m) {
+        const int dyi = (v.cm ? jbase : jbase - m) + pat.ylo;
+        // element e of this window feeds column vv through offset dx = kv*VX + e - vv
+        for (int d = kv * VX - (VX - 1); d <= kv * VX + VX - 1; ++d)
+          for (int vv = 0; vv < VX; ++vv) {
+            const int e = d - kv * VX + vv;
+            if (e < 0 || e >= VX) continue;
+            const int id = cidx(zi, dyi, d + pat.xlo);
+            if (id < 0) continue;
+            if (pair && !(vv & 1) && !(e & 1) && vv + 1 < VX && e + 1 < VX) {
+              f.push_back(fma(id, e, vv, m, zi) | 0x40000000u);   // columns vv, vv+1
+              ++vv;
+              continue;
+            }
+            f.push_back(fma(id, e, vv, m, zi));
           }
+      }
     if (!f.empty()) {
       ops.push_back(load(zsel, j_rel, kv));
       ops.insert(ops.end(), f.begin(), f.end());
@@ -291,7 +314,12 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   o << "__device__ constexpr " << T << " g_coef[" << pat.nnz << "] = {";
   for (int i = 0; i < pat.nnz; ++i) o << hexfloat(pat.c[i], f32) << (i + 1 < pat.nnz ? "," : "");
   o << "};\n";
-  const std::vector<uint32_t> ops = encode_ops(pat, v);
+  // Packed FFMA2 pairs for fp32 are off by default: measured on C3 (star25,
+  // 768^3) they cut FMA instructions by 42% but raise registers 96 -> 151 and
+  // run 2-7% slower (the kernel is not FMA-issue bound).
+  const char* f2 = getenv("STENCIL_FFMA2");                            // dev override
+  const bool pair = f32 && f2 && atoi(f2);
+  const std::vector<uint32_t> ops = encode_ops(pat, v, pair);
   o << "__device__ constexpr unsigned g_ops[" << std::max<size_t>(ops.size(), 1) << "] = {";
   for (size_t i = 0; i < ops.size(); ++i) o << ops[i] << "u" << (i + 1 < ops.size() ? "," : "");
   if (ops.empty()) o << "0u";
@@ -301,7 +329,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   if (v.family == FAM_STREAM_TB) {     // intermediate fused steps: VX x MI tiles, gather or (RT) scatter
     Variant vm = v;
     vm.family = FAM_STREAM; vm.cm = false; vm.m = mi;
-    mops = encode_ops(pat, vm);
+    mops = encode_ops(pat, vm, pair);
   }
   o << "__device__ constexpr unsigned g_mops[" << std::max<size_t>(mops.size(), 1) << "] = {";
   for (size_t i = 0; i < mops.size(); ++i) o << mops[i] << "u" << (i + 1 < mops.size() ? "," : "");
@@ -312,6 +340,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   int minb = 1;   // __launch_bounds__ min blocks of k_stream_tb_rt
   if (const char* e = getenv("STENCIL_MINB")) minb = atoi(e);   // dev override
   o << "  static constexpr int MINB = " << minb << ";\n";
+  o << "  static constexpr int MIDR = " << v.mid_slots() << ";\n";
   o << "  struct Mid {\n    static constexpr int NOPS = " << mops.size() << ";\n"
     << "    static __device__ __forceinline__ constexpr unsigned op(int i) { return g_mops[i]; }\n  };\n";
   o << "  static constexpr int NNZ = " << pat.nnz << ", ZLO = " << pat.zlo << ", ZHI = " << pat.zhi

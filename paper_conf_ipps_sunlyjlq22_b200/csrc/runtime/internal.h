@@ -86,6 +86,7 @@ struct Variant {
   int threads() const;
   int smem_bytes(const Pattern& p, int elem) const;
   int mid_rows(const Pattern& p, int elem) const;
+  int mid_slots() const;
   int tbrt_threads(const Pattern& p, int elem) const;
 };
 
