@@ -257,3 +257,22 @@ def test_tb_rt_pipeline_settings(gpu, name, dims, dtype):
         assert np.array_equal(got, base), (oc, prm)
         ran += 1
     assert ran >= 3
+
+
+@pytest.mark.parametrize("name,dims,dtype,oc,prm", [
+    ("heat3d", (20, 100, 200), "f64", "ST_TB_BM_RT_PR", None),
+    ("heat3d", (21, 90, 170), "f64", "ST_TB_CM_RT", {"merge": 4, "by": 4}),
+    ("star25", (24, 80, 300), "f32", "ST_TB_RT_PR", None),
+    ("random3d:2:5", (22, 70, 140), "f64", "ST_TB_BM_RT_PR", {"tb_steps": 3, "merge": 2})])
+def test_tb_rt_interior_and_edge_tiles(gpu, name, dims, dtype, oc, prm):
+    """k_stream_tb_rt on grids large enough that some tiles lie wholly inside
+    the compute box next to edge tiles (frame values of the intermediate step
+    come from the input ring); element-wise vs the oracle, bitwise vs OC base."""
+    acc, c = si.config_stencil(name)
+    steps = 4
+    u0 = si.make_field(dims, 31, dtype)
+    ref = oracle.sweep(u0, acc, c, steps, dtype=dtype)
+    base = _run(sm.Plan(dims, acc, c, dtype, 0), u0, dtype, steps)
+    got = _run(sm.Plan(dims, acc, c, dtype, sm.oc_from_name(oc), prm), u0, dtype, steps)
+    assert _relerr(got, ref) <= TOL[dtype]
+    assert np.array_equal(got, base)
