@@ -90,11 +90,19 @@ def pearson(x: Sequence[float], y: Sequence[float]) -> float:
     n = len(x)
     if n < 3:
         return 0.0
-    mx = sum(x) / n
-    my = sum(y) / n
-    sxy = sum((a - mx) * (b - my) for a, b in zip(x, y))
-    sxx = sum((a - mx) ** 2 for a in x)
-    syy = sum((b - my) ** 2 for b in y)
+    # plain left-to-right loops (Python's sum() of floats is compensated since 3.12)
+    mx = 0.0
+    my = 0.0
+    for a, b in zip(x, y):
+        mx += a
+        my += b
+    mx /= n
+    my /= n
+    sxy = sxx = syy = 0.0
+    for a, b in zip(x, y):
+        sxy += (a - mx) * (b - my)
+        sxx += (a - mx) * (a - mx)
+        syy += (b - my) * (b - my)
     if sxx == 0.0 or syy == 0.0:
         return 0.0
     return sxy / math.sqrt(sxx * syy)
