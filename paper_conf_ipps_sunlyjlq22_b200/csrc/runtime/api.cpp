@@ -56,7 +56,8 @@ int get_driver(const Driver** out) {
               entry("cuFuncSetAttribute", &g_drv.funcSetAttribute) &&
               entry("cuFuncGetAttribute", &g_drv.funcGetAttribute) && entry("cuLaunchKernel", &g_drv.launchKernel) &&
               entry("cuTensorMapEncodeTiled", &g_drv.tensorMapEncodeTiled) &&
-              entry("cuGetErrorString", &g_drv.getErrorString);
+              entry("cuGetErrorString", &g_drv.getErrorString) &&
+              entry("cuOccupancyMaxActiveBlocksPerMultiprocessor", &g_drv.occupancy);
     g_drv_state = ok ? 1 : -1;
   }
   if (g_drv_state != 1) SM_FAIL(STENCIL_E_CUDA, "CUDA driver entry points unavailable (no GPU driver?)");
@@ -285,7 +286,8 @@ static int resolve_variant(stencil_plan_s* P) {
   if (fam == FAM_TILED || fam == FAM_STREAM || fam == FAM_STREAM_TB) {
     const TmaBox b = tma_box(v, P->pat, elem);
     const bool rows_ok = (P->vdims[2] * elem) % 16 == 0;
-    v.tma = rows_ok && b.lx <= 256 && b.ly <= 256 && b.lz <= 256 && getenv("STENCIL_NO_TMA") == nullptr;
+    const char* notma = getenv("STENCIL_NO_TMA");   // dev / test override: cp.async staging
+    v.tma = rows_ok && b.lx <= 256 && b.ly <= 256 && b.lz <= 256 && !(notma && atoi(notma));
   }
   if (fam == FAM_STREAM_TB && !v.tma)
     SM_FAIL(STENCIL_E_OC_INFEASIBLE, "OC %s needs TMA staging (rows of 16-byte multiples, box <= 256)",
@@ -381,8 +383,28 @@ static int get_tmap(stencil_plan_s* P, const Variant& v, const void* buf, CUtens
   return STENCIL_OK;
 }
 
-static int auto_chunk(const stencil_plan_s* P, const Variant& v, int czlen, long long tiles_xy) {
+// Default z-chunk of the streaming kernels (concurrent streaming).
+// Columns that cannot fill the GPU (2-D grids stream along y with a single
+// row of CTAs per x-tile: 64 tiles at 8192^2) are cut so that about one wave
+// of CTAs is resident, counting at most 16 CTAs per SM: measured on the N2
+// 2-D stencils (8192^2 fp64), chunks of ~200 rows run 1.2-1.3x faster than
+// 512 (too few CTAs) and than 64-128 on order-1 stencils (too many concurrent
+// streams). Otherwise: enough CTAs for ~8 per SM, chunks of at least 16
+// planes (halo reuse); measured on C2, full-depth columns beat any split.
+static int auto_chunk(const stencil_plan_s* P, const Variant& v, const Kernel& k, int threads, int smem,
+                      int czlen, long long tiles_xy) {
   if (v.chunk > 0) return std::min(v.chunk, czlen);
+  int nsm = 0, dev = 0, occ = 0;
+  const Driver* d = nullptr;
+  if (cudaGetDevice(&dev) == cudaSuccess &&
+      cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && get_driver(&d) == 0 &&
+      d->occupancy(&occ, k.fn, threads, (size_t)smem) == CUDA_SUCCESS && occ > 0) {
+    const long long slots = (long long)nsm * std::min(occ, 16);
+    if (tiles_xy * 2 < slots) {
+      const long long nch = std::max(1LL, slots / tiles_xy);
+      return std::min(czlen, std::max(32, (int)((czlen + nch - 1) / nch)));
+    }
+  }
   // enough CTAs for ~8 per SM, but chunks of at least 16 planes (halo reuse)
   long long target = 148LL * 8;
   int c = 1;
@@ -431,7 +453,7 @@ static int launch_sweep(stencil_plan_s* P, const Variant& v, const Kernel& k, co
       args[3] = tm ? (void*)tm : (void*)&dummy;
       nargs = 4;
     } else {
-      chunk = auto_chunk(P, v, czlen, (long long)gx * gy);
+      chunk = auto_chunk(P, v, k, (int)(bx * by), v.smem_bytes(P->pat, elem), czlen, (long long)gx * gy);
       gz = (czlen + chunk - 1) / chunk;
       args[3] = (void*)&chunk;
       args[4] = tm ? (void*)tm : (void*)&dummy;

@@ -55,6 +55,7 @@ struct Driver {
                                    const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
                                    CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
   CUresult (*getErrorString)(CUresult, const char**);
+  CUresult (*occupancy)(int*, CUfunction, int, size_t);   // cuOccupancyMaxActiveBlocksPerMultiprocessor
 };
 int get_driver(const Driver** out);
 const char* cu_errstr(CUresult r);
