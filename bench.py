@@ -554,7 +554,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5", "N2"])
     ap.add_argument("--settings", type=int, default=None,
-                    help="settings per OC in the label pass (default 2; 1 for the multi-stencil C5/N2)")
+                    help="settings per OC in the label pass (default 3; C5: 1, N2: 2)")
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--oc", default="", help="time this OC (skips the label pass); for profiling")
     ap.add_argument("--params", default="", help="JSON parameter setting for --oc")
@@ -566,7 +566,7 @@ def main():
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
     if args.settings is None:
-        args.settings = 1 if args.config in ("C5", "N2") else 2
+        args.settings = {"C5": 1, "N2": 2}.get(args.config, 3)
     if args.impl == "reference":
         return run_reference(args)
     return run_impl(args)
