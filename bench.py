@@ -64,6 +64,15 @@ WORKLOADS = {
 }
 
 
+def _free_port() -> int:
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
 def _env_rank():
     return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
 
@@ -377,6 +386,7 @@ def run_impl(args):
 
     # ---- 1. label pass per stencil: every OC of the family, seeded settings (a8)
     ocs = _ocs_for(name, sm)
+    p2p_flags, p2p_links = None, []
     if args.oc:
         ocs = [sm.oc_from_name(args.oc)]
     t_sw = time.time()
@@ -415,8 +425,20 @@ def run_impl(args):
             best_oc, best_p = obj
         it["per_oc"], it["best_oc"] = per_oc, best_oc
         del base_plan
-        it["plan"] = make_plan(it["acc"], it["c"], best_oc, best_p or None)
-        it["plan"].use_workspace(ws)
+        if slab and args.transport == "p2p":
+            # fused device-initiated halo: edge kernels store the neighbours'
+            # ghost planes through peer memory (CUDA IPC), epochs in flag words
+            from paper_conf_ipps_sunlyjlq22_b200 import p2p
+            if p2p_flags is None:
+                p2p_flags = p2p.new_flags(dev)
+                if world == 1 and not dist.is_initialized():
+                    dist.init_process_group("gloo", init_method="tcp://127.0.0.1:%d" % _free_port(), rank=0,
+                                            world_size=1)
+            it["plan"] = sm.Plan(dims, it["acc"], it["c"], dtype, best_oc, best_p or None)
+            p2p_links.append(p2p.setup_p2p(it["plan"], x, y, ws, p2p_flags, rank, world))
+        else:
+            it["plan"] = make_plan(it["acc"], it["c"], best_oc, best_p or None)
+            it["plan"].use_workspace(ws)
         it["pinfo"] = it["plan"].info
     sweep_s = time.time() - t_sw
     pts_rank = sum(it["points"] for it in items)
@@ -516,7 +538,10 @@ def run_impl(args):
                        else {it["stencil"]: sm.oc_name(it["best_oc"]) for it in items},
                        "params": first["pinfo"]["params"] if len(items) == 1
                        else {it["stencil"]: it["pinfo"]["params"] for it in items},
-                       "parallelism": (f"z-slabs x{world}, NCCL halo exchange (ghost {G} planes), edge/interior overlap"
+                       "parallelism": (f"z-slabs x{world}, "
+                                       + ("fused P2P halo (edge kernels store into peer ghost planes)"
+                                          if args.transport == "p2p" else "NCCL halo exchange")
+                                       + f" (ghost {G} planes), edge/interior overlap"
                                        if slab else "single GPU"),
                        "l2": "inputs (grid bytes) larger than the 126 MB L2; no flush needed"},
             "roofline": roofline,
@@ -562,6 +587,9 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--slab", action="store_true", help="use the NCCL slab path even at N = 1")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p"],
+                    help="halo exchange of the timed slab runs: NCCL send/recv on a comm stream, or the fused "
+                         "device-initiated P2P halo (edge kernels store into the neighbours' ghost planes)")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")

@@ -322,6 +322,45 @@ int stencil_plans_link_loopback(stencil_plan_t *plans, int nranks);
 int stencil_run_group(stencil_plan_t *plans, int nplans, const void *const *ins, void *const *outs,
                       int steps);
 
+/* Fused device-initiated halo (not in the paper): the "P2P"
+ * transport. Instead of NCCL send/recv after the edge kernels, the edge
+ * kernels themselves store each output plane that a neighbour needs into that
+ * neighbour's ghost planes through peer memory (NVLink P2P stores issued tile
+ * by tile with the local stores), then a one-thread kernel publishes an epoch
+ * with a system-scope release store into the neighbour's flag word; before its
+ * next edge kernels a rank waits (acquire loads) until both neighbours have
+ * published that epoch. No NCCL kernel, no comm stream, no staging copy.
+ *   self  this rank's registered grids: stencil_run(plan, in, out, ...) must be
+ *         called with in == self->in, out == self->out and the workspace set to
+ *         self->ws (the neighbours write into their ghost planes);
+ *   lo/hi rank-1 / rank+1 (NULL at the global faces): their registered grids
+ *         and flag words, mapped into this process (stencil_ipc_open_handle, or
+ *         plain pointers for plans of one process);
+ *   flags 16 bytes of device memory per rank (flags[0] is written by rank-1,
+ *         flags[1] by rank+1), zeroed by the caller before any rank registers;
+ *         one flag buffer serves every plan of the rank (epochs are counted
+ *         per flag buffer, so all ranks must run the same sequence of runs);
+ *   owned_planes  the rank's dims[0].
+ * Slab layout, ghost depth and edge/interior split as stencil_plan_set_comm.
+ * stencil_oc_sweep needs an NCCL communicator (E_STATE with this transport). */
+typedef struct {
+    void *in, *out, *ws;
+    uint32_t *flags;
+    int64_t owned_planes;
+} stencil_p2p_buffers_t;
+
+int stencil_plan_set_p2p(stencil_plan_t plan, int rank, int nranks, const stencil_p2p_buffers_t *self,
+                         const stencil_p2p_buffers_t *lo, const stencil_p2p_buffers_t *hi);
+
+/* CUDA IPC for the P2P transport (one process per GPU): the handle of the
+ * allocation that contains dev_ptr (64 bytes) and dev_ptr's byte offset in it;
+ * open maps a peer's allocation into this process and returns the address of
+ * the same byte (base + offset); close unmaps it (pass what open returned and
+ * the same offset). */
+int stencil_ipc_get_handle(const void *dev_ptr, uint8_t *handle, int64_t *offset);
+int stencil_ipc_open_handle(const uint8_t *handle, int64_t offset, void **dev_ptr);
+int stencil_ipc_close(void *dev_ptr, int64_t offset);
+
 /* G, the ghost planes on each side of the plan's slab (0 without a communicator). */
 int stencil_plan_ghost_planes(stencil_plan_t plan);
 

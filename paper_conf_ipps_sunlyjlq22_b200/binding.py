@@ -71,6 +71,12 @@ class SweepRow(ctypes.Structure):
                 ("time_ms", ctypes.c_float)]
 
 
+class P2PBuffers(ctypes.Structure):
+    """stencil_p2p_buffers_t: a rank's registered grids + flag words (device addresses)."""
+    _fields_ = [("in_", ctypes.c_void_p), ("out", ctypes.c_void_p), ("ws", ctypes.c_void_p),
+                ("flags", ctypes.c_void_p), ("owned_planes", ctypes.c_int64)]
+
+
 _lib = None
 
 _SIGS = {
@@ -81,6 +87,11 @@ _SIGS = {
     "stencil_oc_analysis": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_int,
                                            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
                                            ctypes.c_void_p, ctypes.c_void_p]),
+    "stencil_plan_set_p2p": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.POINTER(P2PBuffers),
+                                            ctypes.POINTER(P2PBuffers), ctypes.POINTER(P2PBuffers)]),
+    "stencil_ipc_get_handle": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.POINTER(ctypes.c_int64)]),
+    "stencil_ipc_open_handle": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int64, ctypes.POINTER(ctypes.c_void_p)]),
+    "stencil_ipc_close": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int64]),
     "stencil_plan_create": (ctypes.c_int, [ctypes.POINTER(ctypes.c_void_p), ctypes.c_int,
                                            ctypes.POINTER(ctypes.c_int64), ctypes.c_int, ctypes.c_void_p,
                                            ctypes.c_void_p, ctypes.c_int, ctypes.c_uint32,
@@ -462,9 +473,42 @@ class Plan:
         """Adopt an existing ncclComm_t (e.g. torch's: ProcessGroupNCCL._comm_ptr())."""
         _check(lib().stencil_plan_set_nccl_comm(self._h, ctypes.c_void_p(comm_ptr), rank, nranks))
 
+    def set_p2p(self, rank: int, nranks: int, self_bufs: P2PBuffers, lo: Optional[P2PBuffers],
+                hi: Optional[P2PBuffers]) -> None:
+        """Fused device-initiated halo transport (stencil_plan_set_p2p): the edge
+        kernels store the neighbours' ghost planes through peer memory."""
+        self._p2p = (self_bufs, lo, hi)  # keep the structs alive
+        _check(lib().stencil_plan_set_p2p(self._h, rank, nranks, ctypes.byref(self_bufs),
+                                          ctypes.byref(lo) if lo is not None else None,
+                                          ctypes.byref(hi) if hi is not None else None))
+
     def share_comm(self, other: "Plan") -> None:
         self._comm_src = other          # keep the owner alive
         _check(lib().stencil_plan_share_comm(self._h, other._h))
+
+
+def ipc_handle(ptr: int) -> Tuple[bytes, int]:
+    """CUDA IPC handle (64 bytes) of the allocation holding device address ptr, and ptr's offset in it."""
+    h = (ctypes.c_uint8 * 64)()
+    off = ctypes.c_int64()
+    _check(lib().stencil_ipc_get_handle(ctypes.c_void_p(ptr), h, ctypes.byref(off)))
+    return bytes(h), int(off.value)
+
+
+def ipc_open(handle: bytes, offset: int) -> int:
+    """Map a peer process's allocation; returns the device address of the same byte."""
+    h = (ctypes.c_uint8 * 64).from_buffer_copy(handle)
+    p = ctypes.c_void_p()
+    _check(lib().stencil_ipc_open_handle(h, int(offset), ctypes.byref(p)))
+    return int(p.value)
+
+
+def ipc_close(ptr: int, offset: int) -> None:
+    _check(lib().stencil_ipc_close(ctypes.c_void_p(ptr), int(offset)))
+
+
+def p2p_buffers(inp: int, out: int, ws: int, flags: int, owned_planes: int) -> P2PBuffers:
+    return P2PBuffers(inp, out, ws, flags, owned_planes)
 
 
 def gstencil_per_s(points: int, steps: int, ms: float) -> float:

@@ -41,7 +41,23 @@ struct Grid {
   int uz0, uz1, uy0, uy1, ux0, ux1;  // update box: points inside are updated
   int cz0, cz1, cy0, cy1, cx0, cx1;  // compute box: outputs written by this launch
   int vec_ok;                        // 1 if rows are VX-aligned (vector stores allowed)
+  // P2P halo transport (fused halo): output planes z in
+  // [mlo0, mlo1) are also stored to plane z + shift_lo of the lower
+  // neighbour's buffer peer_lo, planes in [mhi0, mhi1) to plane z + shift_hi of
+  // the upper neighbour's buffer peer_hi (peer memory over NVLink; same
+  // y/x layout). Empty ranges for every launch but the slab-edge ones.
+  long long peer_lo, peer_hi;
+  int mlo0, mlo1, mhi0, mhi1, shift_lo, shift_hi;
 };
+
+// Remote copy of local output plane z (nullptr when z is not mirrored): the
+// address of element `off` of plane z in the neighbour's buffer.
+template <class T>
+__device__ __forceinline__ T* mirror_plane(const Grid& g, int z) {
+  if (z >= g.mlo0 && z < g.mlo1) return reinterpret_cast<T*>(g.peer_lo) + (i64)(z + g.shift_lo) * g.sz;
+  if (z >= g.mhi0 && z < g.mhi1) return reinterpret_cast<T*>(g.peer_hi) + (i64)(z + g.shift_hi) * g.sz;
+  return nullptr;
+}
 
 // ---------------------------------------------------------------------------
 // small PTX helpers
@@ -288,6 +304,7 @@ template <class T, int VX, int M, bool CM, int BYS>
 __device__ __forceinline__ void store_tile(T* __restrict__ out, const Grid& g, int z, int y0, int x0,
                                            const T (&acc)[M][VX]) {
   const bool full_x = (x0 >= g.cx0) && (x0 + VX <= g.cx1) && g.vec_ok;
+  T* const rp = mirror_plane<T>(g, z);
 #pragma unroll
   for (int m = 0; m < M; ++m) {
     const int y = CM ? y0 + m * BYS : y0 + m;
@@ -295,10 +312,14 @@ __device__ __forceinline__ void store_tile(T* __restrict__ out, const Grid& g, i
     T* row = out + z * g.sz + y * g.sy;
     if (full_x) {
       stg_vec<T, VX>(row + x0, acc[m]);
+      if (rp) stg_vec<T, VX>(rp + y * g.sy + x0, acc[m]);
     } else {
 #pragma unroll
       for (int v = 0; v < VX; ++v)
-        if (x0 + v >= g.cx0 && x0 + v < g.cx1) row[x0 + v] = acc[m][v];
+        if (x0 + v >= g.cx0 && x0 + v < g.cx1) {
+          row[x0 + v] = acc[m][v];
+          if (rp) rp[y * g.sy + x0 + v] = acc[m][v];
+        }
     }
   }
 }
@@ -325,8 +346,13 @@ struct TileStore {
       if (y >= g.cy0 && y < g.cy1) rows |= 1u << m;
     }
   }
-  __device__ __forceinline__ void store(int z, const T (&acc)[M][VX]) const {
-    T* p = base + (i64)z * sz;
+  // the same tile also into the neighbour's buffer when plane z is mirrored
+  // (P2P halo transport); `out` is the launch's output grid (kernel parameter)
+  __device__ __forceinline__ void store(int z, const T (&acc)[M][VX], const Grid& g, const T* out) const {
+    store_at(base + (i64)z * sz, acc);
+    if (T* rp = mirror_plane<T>(g, z)) store_at(rp + (base - out), acc);
+  }
+  __device__ __forceinline__ void store_at(T* p, const T (&acc)[M][VX]) const {
     if (full) {
 #pragma unroll
       for (int m = 0; m < M; ++m)
@@ -397,7 +423,10 @@ k_naive(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, G
 #pragma unroll
   for (int m = 0; m < M; ++m) {
     const int y = CM ? y0 + m * BY : y0 + m;
-    if (y < g.cy1) out[(i64)z * g.sz + (i64)y * g.sy + x] = acc[m][0];
+    if (y < g.cy1) {
+      out[(i64)z * g.sz + (i64)y * g.sy + x] = acc[m][0];
+      if (T* rp = mirror_plane<T>(g, z)) rp[(i64)y * g.sy + x] = acc[m][0];
+    }
   }
 }
 
@@ -644,7 +673,7 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
       SmemPlane<T, VX, C::LX> pl{ring + (it % C::NRING) * C::PLANE + row0 * C::LX + col0};
       run_scatter<S, VX, M, NZ - 1>(pl, acc);           // slice zi -> acc[NZ-1-zi]
       const int z = pfirst + it - S::ZHI;               // output completed by this plane
-      if (z >= zs) ts.store(z, acc[0]);
+      if (z >= zs) ts.store(z, acc[0], g, out);
       shift_queue<T, NZ, M, VX>(acc);
       __syncthreads();                                  // slot it%NRING may be refilled
     }
@@ -666,7 +695,7 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
           SmemPlane<T, VX, C::LX> pl{ring + (it % C::NRING) * C::PLANE + row0 * C::LX + col0};
           run_scatter<S, VX, M, U>(pl, acc);
           const int z = pfirst + it - S::ZHI;             // output completed by this plane
-          if (z >= zs) ts.store(z, acc[(U + 1) % NZ]);
+          if (z >= zs) ts.store(z, acc[(U + 1) % NZ], g, out);
           __syncthreads();                                // slot it%NRING may be refilled
         }
       });
@@ -686,7 +715,7 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
         for (int zi = 0; zi < NZ; ++zi)                  // plane z + zi - ZLO
           pl[zi].p = ring + ((it - (NZ - 1) + zi) % C::NRING) * C::PLANE + row0 * C::LX + col0;
         run_gather<S, VX, M>(pl, acc);
-        ts.store(z, acc);
+        ts.store(z, acc, g, out);
       }
       __syncthreads();                                    // oldest slot may be refilled
     }
@@ -1167,7 +1196,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         }
         mbar_arrive(&ein[si]);
         const int z = pin0 + j - TT * S::ZHI;
-        if (act && z >= zs) ts.store(z, acc[(U + 1) % NZ]);
+        if (act && z >= zs) ts.store(z, acc[(U + 1) % NZ], g, out);
         if constexpr (S::RTSHIFT) shift_queue<T, NZ, M, VX>(acc);
       });
     }

@@ -83,6 +83,29 @@ __global__ void k_fill(T* __restrict__ dst, long long bz, long long by, long lon
   }
 }
 
+// P2P transport (fused halo): publish / await an epoch in neighbours' flag
+// words. The signal runs after the edge kernels in stream order; its
+// system-scope fence + release store makes their peer stores visible before
+// the flag. The wait spins on acquire loads (one thread, sleeping between
+// polls) so that later kernels on the stream see the neighbours' planes.
+__global__ void k_p2p_signal(unsigned* a, unsigned* b, unsigned v) {
+  __threadfence_system();
+  if (a) asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(a), "r"(v) : "memory");
+  if (b) asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(b), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ unsigned ld_acquire_sys(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+__global__ void k_p2p_wait(const unsigned* a, const unsigned* b, unsigned v) {
+  // epochs grow monotonically (wrap-safe comparison)
+  if (a) while ((int)(ld_acquire_sys(a) - v) < 0) __nanosleep(128);
+  if (b) while ((int)(ld_acquire_sys(b) - v) < 0) __nanosleep(128);
+}
+
 int grid_for(long long n) {
   long long b = (n + 255) / 256;
   const long long cap = 148LL * 16;
@@ -119,6 +142,22 @@ int launch_fill(void* dst, int dtype, const int64_t box[3], const int64_t org[3]
   else
     k_fill<float><<<grid_for(n), 256, 0, s>>>((float*)dst, box[0], box[1], box[2], org[0], org[1],
                                                org[2], gdim[1], gdim[2], key, kind);
+  g_launches.fetch_add(1);
+  SM_CUDA(cudaGetLastError());
+  return STENCIL_OK;
+}
+
+int launch_p2p_signal(uint32_t* a, uint32_t* b, uint32_t v, cudaStream_t s) {
+  if (!a && !b) return STENCIL_OK;
+  k_p2p_signal<<<1, 1, 0, s>>>(a, b, v);
+  g_launches.fetch_add(1);
+  SM_CUDA(cudaGetLastError());
+  return STENCIL_OK;
+}
+
+int launch_p2p_wait(const uint32_t* a, const uint32_t* b, uint32_t v, cudaStream_t s) {
+  if (!a && !b) return STENCIL_OK;
+  k_p2p_wait<<<1, 1, 0, s>>>(a, b, v);
   g_launches.fetch_add(1);
   SM_CUDA(cudaGetLastError());
   return STENCIL_OK;

@@ -607,6 +607,7 @@ static int run_group(const std::vector<stencil_plan_s*>& Ps, const std::vector<c
   }
   const int T = P0->var.family == FAM_TILED || P0->var.family == FAM_STREAM_TB ? P0->var.tt : 1;
   const int launches = (steps + T - 1) / T;
+  const bool p2p = slab && P0->comm->transport == TR_P2P;
   std::vector<GridArg> gs(np);
   for (size_t k = 0; k < np; ++k) {
     stencil_plan_s* P = Ps[k];
@@ -614,13 +615,46 @@ static int run_group(const std::vector<stencil_plan_s*>& Ps, const std::vector<c
     const size_t bytes = (size_t)P->vdims[0] * P->vdims[1] * P->vdims[2] * elem;
     if (launches >= 2 && (!P->ws || P->ws_bytes < bytes))
       SM_FAIL(STENCIL_E_STATE, "steps=%d needs a workspace of %zu bytes (stencil_plan_set_workspace)", steps, bytes);
+    if (p2p) {
+      const Comm* c = P->comm;
+      if (c->transport != TR_P2P || ins[k] != c->self.in || outs[k] != c->self.out ||
+          (launches >= 2 && P->ws != c->self.ws))
+        SM_FAIL(STENCIL_E_STATE, "P2P slab plans run on their registered in/out/workspace buffers");
+    }
     SM_TRY(ensure_loaded(P));
     gs[k] = make_grid(P, P->var.vx);
+    if (p2p) continue;   // frame copy after the initial halo (below)
     // a4: frame of the input into every buffer the sweep writes (fixed thereafter)
     SM_TRY(launch_frame_copy(ins[k], outs[k], elem, gs[k], P->stream));
     if (launches >= 2) SM_TRY(launch_frame_copy(ins[k], P->ws, elem, gs[k], P->stream));
   }
-  if (slab) {   // ghosts of the input: neighbours' current owned planes
+  if (p2p) {
+    // initial ghosts of `in`: push my edge planes into the neighbours' `in`
+    // ghosts (whole planes, peer memory), publish, await theirs; then the
+    // frame copy (ghost planes included) reads complete planes
+    const int tl0 = std::min(T, steps);
+    for (size_t k = 0; k < np; ++k) {
+      stencil_plan_s* P = Ps[k];
+      Comm* c = P->comm;
+      const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+      const size_t pb = (size_t)P->vdims[1] * P->vdims[2] * elem;
+      const int G = P->ghost, n = (int)P->dims[0];
+      const int up = tl0 * P->pat.zhi, down = tl0 * P->pat.zlo;
+      if (c->has_lo && up)
+        SM_CUDA(cudaMemcpyAsync((char*)c->lo.in + (G + c->lo.owned_planes) * pb, (const char*)ins[k] + G * pb,
+                                up * pb, cudaMemcpyDeviceToDevice, P->stream));
+      if (c->has_hi && down)
+        SM_CUDA(cudaMemcpyAsync((char*)c->hi.in + (G - down) * pb, (const char*)ins[k] + (G + n - down) * pb,
+                                down * pb, cudaMemcpyDeviceToDevice, P->stream));
+      const uint32_t e = ++*p2p_epoch(c->self.flags);
+      SM_TRY(launch_p2p_signal(c->has_lo ? c->lo.flags + 1 : nullptr, c->has_hi ? c->hi.flags : nullptr, e,
+                               P->stream));
+      SM_TRY(launch_p2p_wait(c->has_lo ? c->self.flags : nullptr, c->has_hi ? c->self.flags + 1 : nullptr, e,
+                             P->stream));
+      SM_TRY(launch_frame_copy(ins[k], outs[k], elem, gs[k], P->stream));
+      if (launches >= 2) SM_TRY(launch_frame_copy(ins[k], P->ws, elem, gs[k], P->stream));
+    }
+  } else if (slab) {   // ghosts of the input: neighbours' current owned planes
     std::vector<void*> b(np);
     for (size_t k = 0; k < np; ++k) {
       b[k] = const_cast<void*>(ins[k]);
@@ -642,7 +676,46 @@ static int run_group(const std::vector<stencil_plan_s*>& Ps, const std::vector<c
       if (tl == T) { vs[k] = Ps[k]->var; ks[k] = Ps[k]->kern; }
       else SM_TRY(get_tb_rem_kernel(Ps[k], tl, &vs[k], &ks[k]));
     }
-    if (slab && more) {
+    if (p2p && more) {
+      // fused halo: edge kernels also store the planes the neighbours need
+      // into their ghost planes (same parity buffer), publish, compute the
+      // interior, then await the neighbours before the next launch
+      const int E = tl_next * std::max(P0->pat.zlo, P0->pat.zhi);
+      const bool to_out = (launches - 1 - i) % 2 == 0;
+      for (size_t k = 0; k < np; ++k) {
+        stencil_plan_s* P = Ps[k];
+        Comm* c = P->comm;
+        const int G = P->ghost, n = (int)P->dims[0];
+        GridArg g = gs[k];
+        if (c->has_lo) {
+          g.peer_lo = (long long)(uintptr_t)(to_out ? c->lo.out : c->lo.ws);
+          g.mlo0 = G; g.mlo1 = G + tl_next * P->pat.zhi; g.shift_lo = (int)c->lo.owned_planes;
+        }
+        if (c->has_hi) {
+          g.peer_hi = (long long)(uintptr_t)(to_out ? c->hi.out : c->hi.ws);
+          g.mhi0 = G + n - tl_next * P->pat.zlo; g.mhi1 = G + n; g.shift_hi = -n;
+        }
+        const int c0 = g.cz0, c1 = g.cz1;
+        if (c1 - c0 > 2 * E) {
+          g.cz1 = c0 + E;
+          SM_TRY(launch_sweep(P, vs[k], ks[k], src[k], dst[k], g));
+          g.cz0 = c1 - E; g.cz1 = c1;
+          SM_TRY(launch_sweep(P, vs[k], ks[k], src[k], dst[k], g));
+        } else {
+          SM_TRY(launch_sweep(P, vs[k], ks[k], src[k], dst[k], g));
+        }
+        const uint32_t e = ++*p2p_epoch(c->self.flags);
+        SM_TRY(launch_p2p_signal(c->has_lo ? c->lo.flags + 1 : nullptr, c->has_hi ? c->hi.flags : nullptr, e,
+                                 P->stream));
+        GridArg gi = gs[k];
+        if (gi.cz1 - gi.cz0 > 2 * E) {
+          gi.cz0 += E; gi.cz1 -= E;
+          SM_TRY(launch_sweep(P, vs[k], ks[k], src[k], dst[k], gi));
+        }
+        SM_TRY(launch_p2p_wait(c->has_lo ? c->self.flags : nullptr, c->has_hi ? c->self.flags + 1 : nullptr, e,
+                               P->stream));
+      }
+    } else if (slab && more) {
       const int E = tl_next * std::max(P0->pat.zlo, P0->pat.zhi);
       for (size_t k = 0; k < np; ++k) {   // edge planes first
         GridArg g = gs[k];

@@ -124,6 +124,12 @@ static int slab_setup(stencil_plan_s* P, int rank, int nranks, int transport) {
   return STENCIL_OK;
 }
 
+namespace smart_rt {
+int slab_setup_ext(stencil_plan_s* P, int rank, int nranks, int transport) {
+  return slab_setup(P, rank, nranks, transport);
+}
+}  // namespace smart_rt
+
 extern "C" int stencil_nccl_unique_id(uint8_t* id) {
   clear_error();
   if (!id) SM_FAIL(STENCIL_E_INVAL, "null id");

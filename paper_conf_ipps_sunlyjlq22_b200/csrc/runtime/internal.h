@@ -112,6 +112,8 @@ struct GridArg {
   int uz0, uz1, uy0, uy1, ux0, ux1;
   int cz0, cz1, cy0, cy1, cx0, cx1;
   int vec_ok;
+  long long peer_lo, peer_hi;                     // P2P: mirror stores (layout of smart::Grid)
+  int mlo0, mlo1, mhi0, mhi1, shift_lo, shift_hi;
 };
 
 // AOT kernels (aot_kernels.cu)
@@ -125,7 +127,7 @@ int launch_fill(void* dst, int dtype, const int64_t box[3], const int64_t org[3]
 // by G more: the device array has n + 2G planes. Transport: NCCL send/recv
 // between processes, or LOOPBACK (all slabs as plans of one process, halos by
 // cudaMemcpyAsync -- the multi-GPU schedule exercised on one device).
-enum Transport { TR_NONE = 0, TR_NCCL = 1, TR_LOOPBACK = 2 };
+enum Transport { TR_NONE = 0, TR_NCCL = 1, TR_LOOPBACK = 2, TR_P2P = 3 };
 
 struct Comm {
   int transport = TR_NONE;
@@ -137,7 +139,14 @@ struct Comm {
   cudaEvent_t ev_comm = nullptr;     // halo exchange into dst done (comm stream)
   std::vector<stencil_plan_s*> peers;  // LOOPBACK: plans of all ranks (index = rank)
   const void* cur = nullptr;         // LOOPBACK: buffer this rank is exchanging (for peers)
+  // P2P (fused halo): registered grids of this rank and its neighbours
+  stencil_p2p_buffers_t self{}, lo{}, hi{};
+  bool has_lo = false, has_hi = false;
 };
+// P2P transport: epoch counter of a flag buffer (shared by the rank's plans)
+uint32_t* p2p_epoch(const void* flags);
+int launch_p2p_signal(uint32_t* flag_a, uint32_t* flag_b, uint32_t v, cudaStream_t s);
+int launch_p2p_wait(const uint32_t* flag_a, const uint32_t* flag_b, uint32_t v, cudaStream_t s);
 void comm_destroy(Comm* c);
 int comm_create_stream_events(Comm* c);
 // Halo plane ranges (local plane indices) of a launch fusing `tl` steps.
