@@ -107,6 +107,13 @@ __device__ __forceinline__ void tma_load_3d(void* dst, const TmaDesc* desc, unsi
       :: "r"(smem_u32(dst)), "l"(reinterpret_cast<unsigned long long>(desc)),
          "r"(x), "r"(y), "r"(z), "r"(smem_u32(bar)) : "memory");
 }
+// warp-role register redistribution (warpgroup-aligned, sm_90a+/sm_100a)
+template <int N> __device__ __forceinline__ void setmaxnreg_dec() {
+  asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" :: "n"(N));
+}
+template <int N> __device__ __forceinline__ void setmaxnreg_inc() {
+  asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" :: "n"(N));
+}
 __device__ __forceinline__ void tma_prefetch_desc(const TmaDesc* desc) {
   asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<unsigned long long>(desc)) : "memory");
 }
@@ -325,19 +332,25 @@ __device__ __forceinline__ void store_tile(T* __restrict__ out, const Grid& g, i
 }
 
 // The same store with the plane-invariant part hoisted: streaming kernels
-// build it once per thread and store one tile per plane.
-template <class T, int VX, int M, bool CM, int BYS>
+// build it once per thread and store one tile per plane. SY / SZ: the row and
+// plane strides baked into the kernel by the generator (S::SY, S::SZ; 0 = take
+// them from the Grid at run time) -- compile-time strides turn the per-plane
+// address arithmetic into immediates (no 64-bit multiplies, no constant-bank
+// reloads in the loop).
+template <class T, int VX, int M, bool CM, int BYS, i64 SY = 0, i64 SZ = 0>
 struct TileStore {
   T* base;             // element (plane 0, row y0, column x0)
-  i64 sz, rs;          // plane stride, stride between the tile's rows
+  i64 sz_, rs_;        // plane stride, stride between the tile's rows (run-time strides)
   unsigned rows;       // bit m: row m inside the compute box
   bool full;           // whole vectors inside the compute box (128-bit stores)
   int x0, cx0, cx1;
+  __device__ __forceinline__ i64 sz() const { return SZ ? SZ : sz_; }
+  __device__ __forceinline__ i64 rs() const { return SY ? (CM ? BYS : 1) * SY : rs_; }
   __device__ __forceinline__ TileStore(T* out, const Grid& g, int y0, int x0_) {
     x0 = x0_; cx0 = g.cx0; cx1 = g.cx1;
-    base = out + (i64)y0 * g.sy + x0;
-    sz = g.sz;
-    rs = (CM ? BYS : 1) * g.sy;
+    base = out + (i64)y0 * (SY ? SY : g.sy) + x0;
+    sz_ = g.sz;
+    rs_ = (CM ? BYS : 1) * g.sy;
     full = (x0 >= g.cx0) && (x0 + VX <= g.cx1) && g.vec_ok;
     rows = 0;
 #pragma unroll
@@ -349,21 +362,21 @@ struct TileStore {
   // the same tile also into the neighbour's buffer when plane z is mirrored
   // (P2P halo transport); `out` is the launch's output grid (kernel parameter)
   __device__ __forceinline__ void store(int z, const T (&acc)[M][VX], const Grid& g, const T* out) const {
-    store_at(base + (i64)z * sz, acc);
+    store_at(base + (i64)z * sz(), acc);
     if (T* rp = mirror_plane<T>(g, z)) store_at(rp + (base - out), acc);
   }
   __device__ __forceinline__ void store_at(T* p, const T (&acc)[M][VX]) const {
     if (full) {
 #pragma unroll
       for (int m = 0; m < M; ++m)
-        if (rows & (1u << m)) stg_vec<T, VX>(p + m * rs, acc[m]);
+        if (rows & (1u << m)) stg_vec<T, VX>(p + m * rs(), acc[m]);
     } else {
 #pragma unroll
       for (int m = 0; m < M; ++m) {
         if (!(rows & (1u << m))) continue;
 #pragma unroll
         for (int v = 0; v < VX; ++v)
-          if (x0 + v >= cx0 && x0 + v < cx1) p[m * rs + v] = acc[m][v];
+          if (x0 + v >= cx0 && x0 + v < cx1) p[m * rs() + v] = acc[m][v];
       }
     }
   }
@@ -655,7 +668,7 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
   const int col0 = C::XOFF + tx * VX;
   const int x0 = xb + tx * VX;
   const int y0 = yb + (CM ? ty : ty * M);
-  const TileStore<T, VX, M, CM, BY> ts(out, g, y0, x0);
+  const TileStore<T, VX, M, CM, BY, S::SY, S::SZ> ts(out, g, y0, x0);
 
   if constexpr (RT && S::RTSHIFT) {
     // large op tables (high-order stencils): one copy of the plane body and a
@@ -1002,8 +1015,14 @@ struct StreamTbRtCfg {
   static constexpr int SMEM = ELEMS * (int)sizeof(T) + 8 * NBAR + 128;
   static constexpr int FT = (BX / VX) * BY;                 // last-stage tiles
   static constexpr int WF = (FT + 31) / 32;
-  static constexpr int WL = TbRtWarp0<S, BX, BY, VX, M, TT, MI, TT>::value;   // first last-stage warp
-  static constexpr int THREADS = 32 * (WL + WF);
+  // register split (S::REG_LO > 0): producer + intermediate stages give
+  // registers to the last stage (setmaxnreg); role boundaries are then
+  // warpgroup-aligned by idle padding warps
+  static constexpr bool SPLIT = S::REG_LO > 0;
+  static constexpr int WL0 = TbRtWarp0<S, BX, BY, VX, M, TT, MI, TT>::value;
+  static constexpr int WL = SPLIT ? (WL0 + 3) / 4 * 4 : WL0;   // first last-stage warp
+  static constexpr int NW = SPLIT ? (WL + WF + 3) / 4 * 4 : WL + WF;
+  static constexpr int THREADS = 32 * NW;
 };
 
 template <class S, int BX, int BY, int VX, int M, bool CM, int NS, int TT>
@@ -1058,6 +1077,10 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
   }
   fence_proxy_async();                                  // generic zero-fill before async-proxy writes
   __syncthreads();
+  if constexpr (C::SPLIT) {
+    if (warp < C::WL) setmaxnreg_dec<S::REG_LO>();
+    else setmaxnreg_inc<S::REG_HI>();
+  }
 
   // ------------------------------------------------------------ producer
   if (warp == 0) {
@@ -1163,7 +1186,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
       });
     }
   });
-  if (done) return;
+  if (done || warp < C::WL || warp >= C::WL + C::WF) return;   // (idle padding warps)
 
   // ------------------------------------------------------------ last stage
   {
@@ -1174,7 +1197,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     const int col0 = C::XOFF + tx * VX;
     const int x0 = xb + tx * VX;
     const int y0 = yb + (CM ? ty : ty * M);
-    const TileStore<T, VX, M, CM, BY> ts(out, g, y0, x0);
+    const TileStore<T, VX, M, CM, BY, S::SY, S::SZ> ts(out, g, y0, x0);
     unsigned long long* fin = full_s(TT - 1);
     unsigned long long* ein = empty_s(TT - 1);
     T acc[NZ][M][VX];

@@ -247,6 +247,36 @@ static TmaBox tma_box(const Variant& v, const Pattern& p, int elem) {
   return {ru(xoff + v.bx + t * p.xhi, aln), v.by * v.m + t * (p.ylo + p.yhi), 1};
 }
 
+// Register split of the warp-specialised ST_TB_RT kernel (setmaxnreg): the
+// CTA runs alone on its SM (__launch_bounds__(THREADS, 1)), so every warp gets
+// the same cap R0 = 64K / THREADS; the producer and intermediate-stage warps
+// shrink to R0 - 8 and the last stage -- the pipeline's slowest stage, which
+// spills at R0 -- grows by what they free. Measured on C2 (512^3 heat, fp64,
+// T = 2, 896 threads, R0 = 72): 517 -> 530 GStencil/s with 64/88, no spills
+// (56/112: 521). Applied only when aligning the roles to warpgroups costs at
+// most 2 idle warps; ensure_loaded() drops the split if the compiled kernel
+// holds fewer registers than the pool needs.
+static void choose_regsplit(Variant* v, const Pattern& pat, int elem) {
+  v->reg_lo = v->reg_hi = 0;
+  if (const char* e = getenv("STENCIL_REGSPLIT")) {   // dev override: "lo,hi" (or "0,0" = off)
+    if (sscanf(e, "%d,%d", &v->reg_lo, &v->reg_hi) != 2) v->reg_lo = v->reg_hi = 0;
+    return;
+  }
+  int wl = 0;
+  const int nw0 = v->tbrt_threads(pat, elem, &wl) / 32;
+  v->reg_lo = 1;                                   // padded (warpgroup-aligned) layout
+  const int nw = v->tbrt_threads(pat, elem, &wl) / 32;
+  v->reg_lo = 0;
+  if (nw * 32 > 1024 || nw > nw0 + 2 || wl >= nw) return;
+  const int r0 = std::min(255, (65536 / (nw * 32)) / 8 * 8);
+  const int lo = r0 - 8;
+  if (lo < 40) return;
+  const int hi = std::min(256, ((nw * r0 - wl * lo) / (nw - wl)) / 8 * 8);
+  if (hi <= r0) return;
+  v->reg_lo = lo;
+  v->reg_hi = hi;
+}
+
 static int resolve_variant(stencil_plan_s* P) {
   const stencil_params_t& p = P->params;
   const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
@@ -273,7 +303,10 @@ static int resolve_variant(stencil_plan_s* P) {
   if (v.m > 8) SM_FAIL(STENCIL_E_INVAL, "merge factor must be <= 8");
   if (v.tt < 1 || v.tt > 8) SM_FAIL(STENCIL_E_INVAL, "tb_steps must be in 1..8");
   if (v.ns < 1 || v.ns > 8) SM_FAIL(STENCIL_E_INVAL, "pr_stages must be in 1..8");
-  if (fam == FAM_STREAM_TB && v.rt && v.tt >= 2) v.ws_threads = v.tbrt_threads(P->pat, elem);
+  if (fam == FAM_STREAM_TB && v.rt && v.tt >= 2) {
+    choose_regsplit(&v, P->pat, elem);
+    v.ws_threads = v.tbrt_threads(P->pat, elem);
+  }
   const int thr = v.threads();
   if (thr < 32 || thr > 1024)
     SM_FAIL(STENCIL_E_OC_INFEASIBLE, "CTA of %d threads outside 32..1024", thr);
@@ -294,6 +327,10 @@ static int resolve_variant(stencil_plan_s* P) {
             oc_name_static(P->oc));
   if (fam == FAM_STREAM_TB && v.tt < 2) v.family = FAM_STREAM;
   v.chunk = p.stream_chunk;
+  v.sy = P->vdims[2];                       // = make_grid's strides (contiguous view)
+  v.sz = P->vdims[1] * P->vdims[2];
+  if (const char* e = getenv("STENCIL_NO_BAKE"))   // dev override: run-time strides
+    if (atoi(e)) v.sy = v.sz = 0;
   P->var = v;
   return STENCIL_OK;
 }
@@ -347,6 +384,18 @@ static int ensure_loaded(stencil_plan_s* P) {
   const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
   if (P->cubin.empty()) SM_TRY(compile_variant(P->pat, P->dtype, P->var, &P->lowered, &P->cubin));
   SM_TRY(load_kernel(P->src, P->cubin, P->lowered, P->var.smem_bytes(P->pat, elem), &P->kern));
+  if (!P->var.regsplit_fits(P->pat, elem, P->kern.regs)) {
+    if (getenv("STENCIL_REGSPLIT"))
+      SM_FAIL(STENCIL_E_OC_INFEASIBLE, "register split %d/%d does not fit %d regs/thread", P->var.reg_lo,
+              P->var.reg_hi, P->kern.regs);
+    // the kernel holds fewer registers than the split needs: recompile without it
+    P->var.reg_lo = P->var.reg_hi = 0;
+    P->var.ws_threads = P->var.tbrt_threads(P->pat, elem);
+    P->src = generate_source(P->pat, P->dtype, P->var);
+    P->cubin.clear();
+    SM_TRY(compile_variant(P->pat, P->dtype, P->var, &P->lowered, &P->cubin));
+    SM_TRY(load_kernel(P->src, P->cubin, P->lowered, P->var.smem_bytes(P->pat, elem), &P->kern));
+  }
   P->loaded = true;
   return STENCIL_OK;
 }
@@ -486,6 +535,7 @@ static int launch_sweep(stencil_plan_s* P, const Variant& v, const Kernel& k, co
 static int get_tb_rem_kernel(stencil_plan_s* P, int tt, Variant* vout, Kernel* kout) {
   Variant v = P->var;
   v.tt = tt;
+  v.reg_lo = v.reg_hi = 0;   // remainder launches are rare: no register split
   if (v.family == FAM_STREAM_TB && tt == 1) v.family = FAM_STREAM;   // remainder of one step: plain ST
   const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
   if (v.family == FAM_STREAM_TB && v.rt) {
@@ -504,6 +554,9 @@ static int get_tb_rem_kernel(stencil_plan_s* P, int tt, Variant* vout, Kernel* k
   SM_TRY(compile_variant(P->pat, P->dtype, v, &low, &bin));
   Kernel k;
   SM_TRY(load_kernel(generate_source(P->pat, P->dtype, v), bin, low, v.smem_bytes(P->pat, elem), &k));
+  if (!v.regsplit_fits(P->pat, elem, k.regs))
+    SM_FAIL(STENCIL_E_OC_INFEASIBLE, "register split %d/%d does not fit %d regs/thread", v.reg_lo, v.reg_hi,
+            k.regs);
   P->tb_rem[tt] = k;
   *kout = k;
   return STENCIL_OK;
@@ -866,6 +919,22 @@ int stencil_plan_create(stencil_plan_t* plan, int ndim, const int64_t* dims, int
     else return rc;
   }
   clear_error();
+  if (P->var.reg_lo > 0 && !getenv("STENCIL_REGSPLIT")) {
+    // keep the register split only where it pays: the unsplit kernel spills,
+    // the CTA is alone on its SM anyway (shared memory), and the split kernel
+    // spills less (large op tables: the intermediate stages need their registers)
+    const int elem = dtype == STENCIL_F64 ? 8 : 4;
+    Variant v0 = P->var;
+    v0.reg_lo = v0.reg_hi = 0;
+    v0.ws_threads = v0.tbrt_threads(P->pat, elem);
+    std::string low;
+    std::vector<char> bin;
+    int sp0 = -1, sp1 = -1;
+    SM_TRY(compile_variant(P->pat, P->dtype, v0, &low, &bin, &sp0));
+    const bool alone = 2 * (v0.smem_bytes(P->pat, elem) + 1024) > 228 * 1024;
+    if (sp0 > 0 && alone) SM_TRY(compile_variant(P->pat, P->dtype, P->var, &low, &bin, &sp1));
+    if (!(sp0 > 0 && alone && sp1 >= 0 && sp1 < sp0)) P->var = v0;
+  }
   P->src = generate_source(P->pat, P->dtype, P->var);
   // kernel specialisation (host-only; module load is deferred to first use)
   SM_TRY(compile_variant(P->pat, P->dtype, P->var, &P->lowered, &P->cubin));

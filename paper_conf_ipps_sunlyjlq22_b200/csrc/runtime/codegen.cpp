@@ -31,6 +31,7 @@ namespace {
 std::mutex g_mu;
 std::map<std::string, CUmodule> g_modules;          // source -> loaded module
 std::map<std::string, std::pair<std::string, std::vector<char>>> g_cubins;  // source -> (lowered, cubin)
+std::map<std::string, int> g_spills;                                          // source -> ptxas spill bytes
 
 uint64_t fnv1a(const std::string& s) {
   uint64_t h = 1469598103934665603ull;
@@ -149,6 +150,25 @@ int Variant::mid_slots() const {
 // Mirrors StreamTbRtCfg::THREADS of stencil_kernels.cuh: one producer warp,
 // ceil(NT_s / 32) warps per intermediate stage s, ceil(tiles / 32) last-stage warps.
 int Variant::tbrt_threads(const Pattern& p, int elem) const {
+  int wl = 0;
+  return tbrt_threads(p, elem, &wl);
+}
+
+// Register split (setmaxnreg) of k_stream_tb_rt: warps [0, WL) shrink to
+// reg_lo, the last stage [WL, NW) grows to reg_hi. The growth is served from
+// the CTA's own allocation (regs/thread of the compiled kernel x NW warps), so
+// the split must fit it -- otherwise setmaxnreg.inc would wait forever. Checked
+// against the loaded kernel's register count before any launch.
+bool Variant::regsplit_fits(const Pattern& p, int elem, int kernel_regs) const {
+  if (reg_lo <= 0) return true;
+  int wl = 0;
+  const int nw = tbrt_threads(p, elem, &wl) / 32;
+  if (reg_lo % 8 || reg_hi % 8 || reg_lo < 24 || reg_hi > 256 || reg_lo > kernel_regs || reg_hi < kernel_regs)
+    return false;
+  return (long)wl * reg_lo + (long)(nw - wl) * reg_hi <= (long)nw * kernel_regs;
+}
+
+int Variant::tbrt_threads(const Pattern& p, int elem, int* wl_out) const {
   const int mi = mid_rows(p, elem);
   int warps = 1;
   for (int s = 1; s < tt; ++s) {
@@ -159,7 +179,10 @@ int Variant::tbrt_threads(const Pattern& p, int elem) const {
     const int nty = (by * m + hy0 + hy1 + mi - 1) / mi;
     warps += (ntx * nty + 31) / 32;
   }
+  if (reg_lo > 0) warps = roundup(warps, 4);    // warpgroup-aligned roles (register split)
+  *wl_out = warps;
   warps += ((bx / vx) * by + 31) / 32;
+  if (reg_lo > 0) warps = roundup(warps, 4);
   return 32 * warps;
 }
 
@@ -341,6 +364,8 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   if (const char* e = getenv("STENCIL_MINB")) minb = atoi(e);   // dev override
   o << "  static constexpr int MINB = " << minb << ";\n";
   o << "  static constexpr int MIDR = " << v.mid_slots() << ";\n";
+  o << "  static constexpr int REG_LO = " << v.reg_lo << ", REG_HI = " << v.reg_hi << ";\n";
+  o << "  static constexpr long long SY = " << v.sy << "LL, SZ = " << v.sz << "LL;   // baked strides\n";
   o << "  struct Mid {\n    static constexpr int NOPS = " << mops.size() << ";\n"
     << "    static __device__ __forceinline__ constexpr unsigned op(int i) { return g_mops[i]; }\n  };\n";
   o << "  static constexpr int NNZ = " << pat.nnz << ", ZLO = " << pat.zlo << ", ZHI = " << pat.zhi
@@ -364,9 +389,27 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   return o.str();
 }
 
+// spill bytes (stores + loads) from the ptxas -v lines of an NVRTC log; -1 if absent
+static int parse_spill(const std::string& log) {
+  int total = -1;
+  size_t pos = 0;
+  while ((pos = log.find("bytes spill stores", pos)) != std::string::npos) {
+    size_t b = log.rfind(',', pos);
+    const int st = b == std::string::npos ? 0 : atoi(log.c_str() + b + 1);
+    const size_t l = log.find("bytes spill loads", pos);
+    size_t b2 = l == std::string::npos ? std::string::npos : log.rfind(',', l);
+    const int ld = b2 == std::string::npos ? 0 : atoi(log.c_str() + b2 + 1);
+    total = std::max(total, 0) + st + ld;
+    pos += 8;
+  }
+  return total;
+}
+
 int compile_variant(const Pattern& pat, int dtype, const Variant& v, std::string* lowered,
-                    std::vector<char>* cubin) {
+                    std::vector<char>* cubin, int* spill_bytes) {
   const std::string src = generate_source(pat, dtype, v);
+  int spill_dummy = 0;
+  if (!spill_bytes) spill_bytes = &spill_dummy;
   const std::string expr = "&" + v.name_expr("gen::S");
   {
     std::lock_guard<std::mutex> lk(g_mu);
@@ -374,11 +417,12 @@ int compile_variant(const Pattern& pat, int dtype, const Variant& v, std::string
     if (it != g_cubins.end()) {
       *lowered = it->second.first;
       *cubin = it->second.second;
+      *spill_bytes = g_spills[src];
       return STENCIL_OK;
     }
   }
   std::vector<const char*> optv = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "-default-device",
-                                   "--extra-device-vectorization"};
+                                   "--extra-device-vectorization", "--ptxas-options=-v"};
   static thread_local std::string maxreg_opt;
   if (const char* e = getenv("STENCIL_MAXRREG")) {   // dev override (register cap experiments)
     maxreg_opt = std::string("--maxrregcount=") + e;
@@ -397,12 +441,14 @@ int compile_variant(const Pattern& pat, int dtype, const Variant& v, std::string
   const std::string base = dir + "/" + hname;
 
   // disk cache
-  std::vector<char> bin, nm;
-  if (read_file(base + ".cubin", &bin) && read_file(base + ".name", &nm)) {
+  std::vector<char> bin, nm, sp;
+  if (read_file(base + ".cubin", &bin) && read_file(base + ".name", &nm) && read_file(base + ".spill", &sp)) {
     *lowered = std::string(nm.begin(), nm.end());
     *cubin = bin;
+    *spill_bytes = atoi(std::string(sp.begin(), sp.end()).c_str());
     std::lock_guard<std::mutex> lk(g_mu);
     g_cubins[src] = {*lowered, *cubin};
+    g_spills[src] = *spill_bytes;
     return STENCIL_OK;
   }
 
@@ -422,6 +468,13 @@ int compile_variant(const Pattern& pat, int dtype, const Variant& v, std::string
     if (log.size() > 3000) log = log.substr(0, 3000) + "...";
     SM_FAIL(STENCIL_E_NVRTC, "NVRTC compile of %s failed: %s", expr.c_str(), log.c_str());
   }
+  {
+    size_t ls = 0;
+    nvrtcGetProgramLogSize(prog, &ls);
+    std::string log(ls, '\0');
+    if (ls) nvrtcGetProgramLog(prog, &log[0]);
+    *spill_bytes = parse_spill(log);
+  }
   const char* low = nullptr;
   nvrtcGetLoweredName(prog, expr.c_str(), &low);
   *lowered = low ? low : "";
@@ -433,10 +486,13 @@ int compile_variant(const Pattern& pat, int dtype, const Variant& v, std::string
   {
     std::lock_guard<std::mutex> lk(g_mu);
     g_cubins[src] = {*lowered, *cubin};
+    g_spills[src] = *spill_bytes;
   }
   mkdirs(dir);
   write_file_atomic(base + ".cubin", cubin->data(), cubin->size());
   write_file_atomic(base + ".name", lowered->data(), lowered->size());
+  const std::string spn = std::to_string(*spill_bytes);
+  write_file_atomic(base + ".spill", spn.data(), spn.size());
   return STENCIL_OK;
 }
 

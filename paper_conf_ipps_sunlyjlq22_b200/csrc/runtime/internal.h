@@ -83,12 +83,16 @@ struct Variant {
   bool tma = false;
   int chunk = 0;         // runtime argument (streaming)
   int ws_threads = 0;    // warp-specialised ST_TB_RT kernel: CTA size (tbrt_threads)
+  long long sy = 0, sz = 0;   // row / plane strides baked into the kernel (0 = run time)
+  int reg_lo = 0, reg_hi = 0; // k_stream_tb_rt register split (setmaxnreg; 0 = off)
   std::string name_expr(const char* desc) const;
   int threads() const;
   int smem_bytes(const Pattern& p, int elem) const;
   int mid_rows(const Pattern& p, int elem) const;
   int mid_slots() const;
   int tbrt_threads(const Pattern& p, int elem) const;
+  int tbrt_threads(const Pattern& p, int elem, int* first_last_warp) const;
+  bool regsplit_fits(const Pattern& p, int elem, int kernel_regs) const;
 };
 
 // Compiled module cache (per process): key = generated source.
@@ -97,8 +101,9 @@ struct Kernel {
   int regs = 0;
   int local_bytes = 0;
 };
+// spill_bytes (optional): ptxas spill stores + loads of the kernel (-1 unknown)
 int compile_variant(const Pattern& pat, int dtype, const Variant& v, std::string* lowered,
-                    std::vector<char>* cubin);
+                    std::vector<char>* cubin, int* spill_bytes = nullptr);
 int load_kernel(const std::string& key_src, const std::vector<char>& cubin, const std::string& lowered,
                 int smem, Kernel* out);
 std::string generate_source(const Pattern& pat, int dtype, const Variant& v);
