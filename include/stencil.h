@@ -107,6 +107,9 @@ typedef struct {
     int32_t uses_tma;         /* 1 if halo tiles are staged with cp.async.bulk.tensor */
     int64_t points;           /* interior points updated per time step (global grid) */
     char kernel_name[128];    /* lowered name of the main kernel */
+    int32_t reg_split[2];     /* warp-specialised ST_TB_RT kernel: registers per thread of the
+                                 producer/intermediate-stage warps and of the last-stage warps
+                                 after setmaxnreg (0, 0 = no split) */
 } stencil_plan_info_t;
 
 /* ---------------------------------------------------------------------------

@@ -58,7 +58,8 @@ class PlanInfo(ctypes.Structure):
                 ("dtype", ctypes.c_int32), ("ext", ctypes.c_int32 * 6), ("oc", ctypes.c_uint32),
                 ("params", Params), ("kernel_family", ctypes.c_int32), ("smem_bytes", ctypes.c_int32),
                 ("threads", ctypes.c_int32), ("regs", ctypes.c_int32), ("uses_tma", ctypes.c_int32),
-                ("points", ctypes.c_int64), ("kernel_name", ctypes.c_char * 128)]
+                ("points", ctypes.c_int64), ("kernel_name", ctypes.c_char * 128),
+                ("reg_split", ctypes.c_int32 * 2)]
 
 
 class Features(ctypes.Structure):
@@ -367,6 +368,7 @@ class Plan:
             "family": FAMILIES[i.kernel_family], "smem_bytes": i.smem_bytes, "threads": i.threads,
             "regs": i.regs, "uses_tma": bool(i.uses_tma), "points": int(i.points),
             "kernel_name": i.kernel_name.decode(),
+            "reg_split": (i.reg_split[0], i.reg_split[1]),
         }
 
     @property

@@ -993,6 +993,8 @@ int stencil_plan_info(stencil_plan_t P, stencil_plan_info_t* info) {
   const GridArg g = make_grid(P, P->var.vx);   // points this plan updates per time step
   info->points = (long long)(g.cz1 - g.cz0) * (g.cy1 - g.cy0) * (g.cx1 - g.cx0);
   snprintf(info->kernel_name, sizeof info->kernel_name, "%s", P->lowered.c_str());
+  info->reg_split[0] = P->var.reg_lo;
+  info->reg_split[1] = P->var.reg_hi;
   return STENCIL_OK;
 }
 

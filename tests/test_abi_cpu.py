@@ -161,3 +161,21 @@ def test_embed_tensor_centred():
     assert np.array_equal(t9[2:7, 2:7, 2:7], acc)
     acc2, _ = si.random_stencil(2, 4, 1)
     assert np.array_equal(sm.embed_tensor(acc2), acc2)
+
+
+def test_tbrt_register_split_choice():
+    """The warp-specialised ST_TB_RT kernel redistributes registers (setmaxnreg)
+    only where it pays: C2's default setting spills at the
+    72-register cap, so its stages shrink to 64 and the last stage grows to 88
+    (20 * 64 + 8 * 88 <= 28 * 72: the growth fits the CTA's own allocation);
+    a setting that does not spill keeps one register count for all warps."""
+    acc, c = si.config_stencil("heat3d")
+    prm = {"bx": 64, "by": 8, "vx": 2, "merge": 4, "tb_steps": 2, "pr_stages": 3}
+    p = _plan((512, 512, 512), acc, c, "f64", sm.oc_from_name("ST_TB_BM_RT_PR"), prm)
+    lo, hi = p.info["reg_split"]
+    assert (lo, hi) == (64, 88) and p.info["threads"] == 896
+    assert 20 * lo + 8 * hi <= 28 * 72
+    q = _plan((512, 512, 512), acc, c, "f64", sm.oc_from_name("ST_TB_RT_PR"))
+    assert q.info["reg_split"] == (0, 0)
+    r = _plan((512, 512, 512), acc, c, "f64", sm.oc_from_name("ST_BM_RT_PR"))
+    assert r.info["reg_split"] == (0, 0)            # only the TB-RT family splits
