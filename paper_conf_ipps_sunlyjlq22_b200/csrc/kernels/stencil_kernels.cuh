@@ -754,7 +754,17 @@ template <class S, int BX, int BY, int VX, int M, bool CM, bool RT, int NS, int 
 struct StreamTbCfg {
   typedef typename S::T T;
   static constexpr int ALN = (16 / (int)sizeof(T)) > VX ? (16 / (int)sizeof(T)) : VX;
-  static constexpr int XOFF = ((TT * S::XLO + ALN - 1) / ALN) * ALN;
+  // Column geometry. Without S::XSHIFT every ring uses the input plane's
+  // geometry (column c = global xb - XOFF + c, XOFF rounded up to ALN). With
+  // S::XSHIFT the ring of step s (s = 0: the TMA input) starts exactly at the
+  // left edge of the region step s+1 needs: xoff(s) = (TT - s) * XLO. A thread
+  // tile of step s+1 then begins XLO columns into its source row, so its
+  // window (XLO left, XHI right) starts on a vector boundary and the op table's
+  // vectors are shifted by XSH = XLO mod VX: a radius-1 fp64 window with VX = 2
+  // is 2 aligned 128-bit loads instead of 3 (one a half-used neighbour vector),
+  // and every output vector still lands aligned in its own ring.
+  static constexpr int XOFF = S::XSHIFT ? TT * S::XLO : ((TT * S::XLO + ALN - 1) / ALN) * ALN;
+  static __device__ __forceinline__ constexpr int xoff(int s) { return S::XSHIFT ? (TT - s) * S::XLO : XOFF; }
   static constexpr int LX = ((XOFF + BX + TT * S::XHI + ALN - 1) / ALN) * ALN;
   static constexpr int LY = BY * M + TT * (S::YLO + S::YHI);
   static constexpr int PLANE = ((LX * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
@@ -980,7 +990,8 @@ template <class S, int BX, int BY, int VX, int M, int TT, int MI, int s>
 struct TbRtStage {
   static constexpr int HX0 = (TT - s) * S::XLO, HX1 = (TT - s) * S::XHI;
   static constexpr int HY0 = (TT - s) * S::YLO, HY1 = (TT - s) * S::YHI;
-  static constexpr int TXL = ((HX0 + VX - 1) / VX) * VX;   // tile x origin = xb - TXL
+  // tile x origin = xb - TXL (S::XSHIFT: exactly the region's left edge, see StreamTbRtCfg)
+  static constexpr int TXL = S::XSHIFT ? HX0 : ((HX0 + VX - 1) / VX) * VX;
   static constexpr int NTX = (TXL + BX + HX1 + VX - 1) / VX;
   static constexpr int RY = BY * M + HY0 + HY1;
   static constexpr int NTY = (RY + MI - 1) / MI;
@@ -1001,7 +1012,17 @@ template <class S, int BX, int BY, int VX, int M, bool CM, int NS, int TT>
 struct StreamTbRtCfg {
   typedef typename S::T T;
   static constexpr int ALN = (16 / (int)sizeof(T)) > VX ? (16 / (int)sizeof(T)) : VX;
-  static constexpr int XOFF = ((TT * S::XLO + ALN - 1) / ALN) * ALN;
+  // Column geometry. Without S::XSHIFT every ring uses the input plane's
+  // geometry (column c = global xb - XOFF + c, XOFF rounded up to ALN). With
+  // S::XSHIFT the ring of step s (s = 0: the TMA input) starts exactly at the
+  // left edge of the region step s+1 needs: xoff(s) = (TT - s) * XLO. A thread
+  // tile of step s+1 then begins XLO columns into its source row, so its
+  // window (XLO left, XHI right) starts on a vector boundary and the op table's
+  // vectors are shifted by XSH = XLO mod VX: a radius-1 fp64 window with VX = 2
+  // is 2 aligned 128-bit loads instead of 3 (one a half-used neighbour vector),
+  // and every output vector still lands aligned in its own ring.
+  static constexpr int XOFF = S::XSHIFT ? TT * S::XLO : ((TT * S::XLO + ALN - 1) / ALN) * ALN;
+  static __device__ __forceinline__ constexpr int xoff(int s) { return S::XSHIFT ? (TT - s) * S::XLO : XOFF; }
   static constexpr int LX = ((XOFF + BX + TT * S::XHI + ALN - 1) / ALN) * ALN;
   static constexpr int LY = BY * M + TT * (S::YLO + S::YHI);
   static constexpr int PLANE = ((LX * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
@@ -1104,12 +1125,14 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     constexpr int W0 = TbRtWarp0<S, BX, BY, VX, M, TT, MI, s>::value;
     if (done || warp < W0 || warp >= W0 + G::W) return;
     done = true;
-    constexpr bool XOVER = C::XOFF - G::TXL + G::NTX * VX > C::LX;
+    constexpr int XO_R = C::xoff(s - 1), XO_W = C::xoff(s);   // source / own ring geometry
+    constexpr bool XOVER = XO_W - G::TXL + G::NTX * VX > C::LX;
     const int t = tid - 32 * W0;
     const bool act = t < G::NT;
     const int gx0 = xb - G::TXL + (t % G::NTX) * VX;
     const int gy0 = yb - G::HY0 + (t / G::NTX) * MI;
-    const int lb = (gy0 - Y0) * C::LX + (gx0 - X0);
+    const int lb_r = (gy0 - Y0) * C::LX + (gx0 - xb + XO_R);   // tile origin in the source ring
+    const int lb = (gy0 - Y0) * C::LX + (gx0 - xb + XO_W);     // ... in the stage's own ring
     const int ry1 = yb + BY * M + G::HY1;
     // rows: bit m = writable (inside R_s rows and the array), bit 8+m = inside the update box
     unsigned rows = 0, allup = 1;
@@ -1121,7 +1144,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
       rows |= (wr ? 1u << m : 0u) | (up ? 1u << (8 + m) : 0u);
       allup &= (gy >= ry1 || up) ? 1u : 0u;
     }
-    const bool xfast = gx0 >= g.ux0 && gx0 + VX <= g.ux1 && (!XOVER || gx0 + VX <= X0 + C::LX);
+    const bool xfast = gx0 >= g.ux0 && gx0 + VX <= g.ux1 && (!XOVER || gx0 - xb + XO_W + VX <= C::LX);
     const bool fast = act && xfast && allup;
     unsigned long long* fin = s == 1 ? full_in : full_s(s - 1);
     unsigned long long* ein = s == 1 ? empty_in : empty_s(s - 1);
@@ -1143,7 +1166,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         mbar_wait_sleep(&fin[si], (unsigned)((j / DIN) & 1));
         if constexpr (!S::RTSHIFT) zero_acc<T, VX, MI>(acc[U]);   // a new output plane starts
         if (act) {
-          SmemPlane<T, VX, C::LX> pl{src + lb};
+          SmemPlane<T, VX, C::LX> pl{src + lb_r - S::XSH};
           run_scatter_ops<S, typename S::Mid, VX, MI, U>(pl, acc);
         }
         if (s > 1) mbar_arrive(&ein[si]);                // input slot read (stage 1: below)
@@ -1152,7 +1175,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         if (j >= MR) mbar_wait_sleep(&empty_s(s)[so], (unsigned)((j / MR - 1) & 1));
         const int zo = pin0 + j - s * S::ZHI;            // plane completed now
         // stage 1: input plane zo (= index j - ZHI) is still in the ring
-        const T* fr = ring0 + ((j - S::ZHI + NR) % NR) * C::PLANE + lb;
+        const T* fr = ring0 + ((j - S::ZHI + NR) % NR) * C::PLANE + lb_r;
         const bool zin = zo >= 0 && zo < g.nz;
         const bool zupd = zo >= g.uz0 && zo < g.uz1;
         const T(&res)[MI][VX] = acc[(U + 1) % NZ];
@@ -1173,7 +1196,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
 #pragma unroll
               for (int v = 0; v < VX; ++v) {
                 const int gx = gx0 + v;
-                if (gx < 0 || gx >= g.nx || gx - X0 >= C::LX) continue;
+                if (gx < 0 || gx >= g.nx || gx - xb + XO_W >= C::LX) continue;
                 const bool upd = rowupd && gx >= g.ux0 && gx < g.ux1;
                 d[v] = upd ? res[m][v] : (s == 1 ? fr[m * C::LX + v] : __ldg(frame + gx));
               }
@@ -1194,7 +1217,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     const bool act = q < C::FT;
     const int tx = q % (BX / VX), ty = q / (BX / VX);
     const int row0 = TT * S::YLO + (CM ? ty : ty * M);
-    const int col0 = C::XOFF + tx * VX;
+    const int col0 = C::xoff(TT - 1) + tx * VX - S::XSH;   // window start in the last ring
     const int x0 = xb + tx * VX;
     const int y0 = yb + (CM ? ty : ty * M);
     const TileStore<T, VX, M, CM, BY, S::SY, S::SZ> ts(out, g, y0, x0);

@@ -243,7 +243,7 @@ static TmaBox tma_box(const Variant& v, const Pattern& p, int elem) {
             v.bz + v.tt * (p.zlo + p.zhi)};
   }
   const int t = v.family == FAM_STREAM_TB ? v.tt : 1;   // stream: halo of t time steps
-  const int xoff = ru(t * p.xlo, aln);
+  const int xoff = v.xshift ? t * p.xlo : ru(t * p.xlo, aln);   // mirrors StreamTbRtCfg::XOFF
   return {ru(xoff + v.bx + t * p.xhi, aln), v.by * v.m + t * (p.ylo + p.yhi), 1};
 }
 
@@ -304,6 +304,21 @@ static int resolve_variant(stencil_plan_s* P) {
   if (v.tt < 1 || v.tt > 8) SM_FAIL(STENCIL_E_INVAL, "tb_steps must be in 1..8");
   if (v.ns < 1 || v.ns > 8) SM_FAIL(STENCIL_E_INVAL, "pr_stages must be in 1..8");
   if (fam == FAM_STREAM_TB && v.rt && v.tt >= 2) {
+    // aligned-window ring geometry (StreamTbRtCfg): possible when the shifted
+    // input offset TT*XLO keeps the TMA box start 16-byte aligned; used when it
+    // saves at least 15% of the window loads. Measured on C2 (512^3, fp64, T=2):
+    // Algorithm-1 order-1 stencils 494 -> 537 GStencil/s (loads -20..-30%);
+    // the heat star saves only 9% and spills more: 530 -> 512, so it keeps the
+    // rounded geometry.
+    const int aln = std::max(16 / elem, v.vx);
+    const bool tma_ok = (v.tt * P->pat.xlo) % aln == 0;
+    if (tma_ok && P->pat.xlo % v.vx != 0) {
+      Variant vs = v;
+      vs.xshift = true;
+      const int l0 = count_window_loads(P->pat, elem, v), l1 = count_window_loads(P->pat, elem, vs);
+      v.xshift = l1 <= 0.85 * l0;
+    }
+    if (const char* nx = getenv("STENCIL_XSHIFT")) v.xshift = tma_ok && atoi(nx) != 0;   // dev override
     choose_regsplit(&v, P->pat, elem);
     v.ws_threads = v.tbrt_threads(P->pat, elem);
   }
@@ -536,6 +551,7 @@ static int get_tb_rem_kernel(stencil_plan_s* P, int tt, Variant* vout, Kernel* k
   Variant v = P->var;
   v.tt = tt;
   v.reg_lo = v.reg_hi = 0;   // remainder launches are rare: no register split
+  if (tt < 2) v.xshift = false;
   if (v.family == FAM_STREAM_TB && tt == 1) v.family = FAM_STREAM;   // remainder of one step: plain ST
   const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
   if (v.family == FAM_STREAM_TB && v.rt) {

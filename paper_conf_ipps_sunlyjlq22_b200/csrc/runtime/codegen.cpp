@@ -174,7 +174,7 @@ int Variant::tbrt_threads(const Pattern& p, int elem, int* wl_out) const {
   for (int s = 1; s < tt; ++s) {
     const int hx0 = (tt - s) * p.xlo, hx1 = (tt - s) * p.xhi;
     const int hy0 = (tt - s) * p.ylo, hy1 = (tt - s) * p.yhi;
-    const int txl = roundup(hx0, vx);
+    const int txl = xshift ? hx0 : roundup(hx0, vx);
     const int ntx = (txl + bx + hx1 + vx - 1) / vx;
     const int nty = (by * m + hy0 + hy1 + mi - 1) / mi;
     warps += (ntx * nty + 31) / 32;
@@ -207,7 +207,7 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     return nring * plane * elem + 8 * nring + 128;
   }
   if (family == FAM_STREAM_TB && rt) {   // mirrors StreamTbRtCfg
-    const int xoff = roundup(tt * p.xlo, aln);
+    const int xoff = xshift ? tt * p.xlo : roundup(tt * p.xlo, aln);
     const int lx = roundup(xoff + bx + tt * p.xhi, aln);
     const int ly = by * m + tt * (p.ylo + p.yhi);
     const int plane = roundup(lx * ly * elem, 128) / elem;
@@ -251,7 +251,11 @@ static std::vector<uint32_t> encode_ops(const Pattern& pat, const Variant& v, bo
   const int VX = v.family == FAM_NAIVE ? 1 : v.vx;
   const int M = v.m, BY = v.by;
   const bool scatter = v.rt && (v.family == FAM_STREAM || v.family == FAM_STREAM_TB);
-  const int KLO = -((pat.xlo + VX - 1) / VX), KHI = (VX - 1 + pat.xhi) / VX;
+  // window vector kv covers columns [kv*VX - xsh, kv*VX - xsh + VX) relative to
+  // the thread's first output column (xsh > 0: TB-RT aligned windows, StreamTbRtCfg)
+  const int xsh = v.xshift ? pat.xlo % VX : 0;
+  auto fdiv = [](int a, int b) { return a >= 0 ? a / b : -((-a + b - 1) / b); };
+  const int KLO = fdiv(xsh - pat.xlo, VX), KHI = fdiv(VX - 1 + pat.xhi + xsh, VX);
   auto load = [](int zi, int j, int kv) {
     return (uint32_t)(zi & 15) | ((uint32_t)(j + 128) & 255) << 4 | ((uint32_t)(kv + 8) & 15) << 12;
   };
@@ -267,9 +271,9 @@ static std::vector<uint32_t> encode_ops(const Pattern& pat, const Variant& v, bo
       for (int m = m_lo; m < m_hi; ++m) {
         const int dyi = (v.cm ? jbase : jbase - m) + pat.ylo;
         // element e of this window feeds column vv through offset dx = kv*VX + e - vv
-        for (int d = kv * VX - (VX - 1); d <= kv * VX + VX - 1; ++d)
+        for (int d = kv * VX - xsh - (VX - 1); d <= kv * VX - xsh + VX - 1; ++d)
           for (int vv = 0; vv < VX; ++vv) {
-            const int e = d - kv * VX + vv;
+            const int e = d - kv * VX + xsh + vv;
             if (e < 0 || e >= VX) continue;
             const int id = cidx(zi, dyi, d + pat.xlo);
             if (id < 0) continue;
@@ -308,6 +312,17 @@ static std::vector<uint32_t> encode_ops(const Pattern& pat, const Variant& v, bo
     }
   }
   return ops;
+}
+
+// Window LOAD entries of a TB-RT variant's two op tables (last stage + the
+// intermediate stages): the shared-memory vector loads per thread tile and plane.
+int count_window_loads(const Pattern& pat, int elem, const Variant& v) {
+  int n = 0;
+  for (uint32_t op : encode_ops(pat, v, false)) n += !(op >> 31);
+  Variant vm = v;
+  vm.family = FAM_STREAM; vm.cm = false; vm.m = v.mid_rows(pat, elem);
+  for (uint32_t op : encode_ops(pat, vm, false)) n += !(op >> 31);
+  return n;
 }
 
 std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
@@ -364,6 +379,8 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   if (const char* e = getenv("STENCIL_MINB")) minb = atoi(e);   // dev override
   o << "  static constexpr int MINB = " << minb << ";\n";
   o << "  static constexpr int MIDR = " << v.mid_slots() << ";\n";
+  o << "  static constexpr bool XSHIFT = " << (v.xshift ? "true" : "false") << ";\n";
+  o << "  static constexpr int XSH = " << (v.xshift ? pat.xlo % std::max(v.vx, 1) : 0) << ";\n";
   o << "  static constexpr int REG_LO = " << v.reg_lo << ", REG_HI = " << v.reg_hi << ";\n";
   o << "  static constexpr long long SY = " << v.sy << "LL, SZ = " << v.sz << "LL;   // baked strides\n";
   o << "  struct Mid {\n    static constexpr int NOPS = " << mops.size() << ";\n"

@@ -85,6 +85,7 @@ struct Variant {
   int ws_threads = 0;    // warp-specialised ST_TB_RT kernel: CTA size (tbrt_threads)
   long long sy = 0, sz = 0;   // row / plane strides baked into the kernel (0 = run time)
   int reg_lo = 0, reg_hi = 0; // k_stream_tb_rt register split (setmaxnreg; 0 = off)
+  bool xshift = false;        // k_stream_tb_rt: per-step ring geometry with aligned windows
   std::string name_expr(const char* desc) const;
   int threads() const;
   int smem_bytes(const Pattern& p, int elem) const;
@@ -107,6 +108,7 @@ int compile_variant(const Pattern& pat, int dtype, const Variant& v, std::string
 int load_kernel(const std::string& key_src, const std::vector<char>& cubin, const std::string& lowered,
                 int smem, Kernel* out);
 std::string generate_source(const Pattern& pat, int dtype, const Variant& v);
+int count_window_loads(const Pattern& pat, int elem, const Variant& v);
 
 // ---------------------------------------------------------------- kernels
 // Grid descriptor passed by value to the NVRTC kernels (layout must match

@@ -263,7 +263,10 @@ def test_tb_rt_pipeline_settings(gpu, name, dims, dtype):
     ("heat3d", (20, 100, 200), "f64", "ST_TB_BM_RT_PR", None),
     ("heat3d", (21, 90, 170), "f64", "ST_TB_CM_RT", {"merge": 4, "by": 4}),
     ("star25", (24, 80, 300), "f32", "ST_TB_RT_PR", None),
-    ("random3d:2:5", (22, 70, 140), "f64", "ST_TB_BM_RT_PR", {"tb_steps": 3, "merge": 2})])
+    ("random3d:2:5", (22, 70, 140), "f64", "ST_TB_BM_RT_PR", {"tb_steps": 3, "merge": 2}),
+    # order-1 Algorithm-1 stencils take the aligned-window ring geometry (xshift)
+    ("random3d:1:0", (20, 100, 200), "f64", "ST_TB_BM_RT_PR", None),
+    ("random3d:1:1", (23, 75, 150), "f64", "ST_TB_CM_RT_PR", {"merge": 2, "by": 8})])
 def test_tb_rt_interior_and_edge_tiles(gpu, name, dims, dtype, oc, prm):
     """k_stream_tb_rt on grids large enough that some tiles lie wholly inside
     the compute box next to edge tiles (frame values of the intermediate step
