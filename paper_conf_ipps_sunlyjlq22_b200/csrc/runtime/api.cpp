@@ -124,7 +124,9 @@ static void default_params(uint32_t oc, int ndim, int dtype, stencil_params_t* p
     p->bx = 32; p->by = merge ? 4 : 8; p->bz = 1; p->vx = 1;
   } else if (fam == FAM_TILED) {
     p->vx = vmax; p->bx = 16 * vmax; p->by = merge ? 4 : 8; p->bz = (oc & STENCIL_OC_TB) ? 4 : 8;
-    if (ndim == 2) p->bz = 1;
+    // 2-D tiles merge 4 rows per thread (measured on N2's order-1 stencil, 8192^2
+    // fp64, TB_BM: merge 4 -> 597 GStencil/s, merge 2 -> 547)
+    if (ndim == 2) { p->bz = 1; if (merge) p->merge = 4; }
   } else if (fam == FAM_STREAM) {
     // wide, shallow tiles: many small CTAs keep more TMA planes in flight per SM
     // (measured on C2: 128x2 fp64 tiles reach 92% of the copy bandwidth)
@@ -586,6 +588,10 @@ using namespace smart_rt;
 
 stencil_plan_s::~stencil_plan_s() {
   for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
+  for (cudaEvent_t e : h2d_ev) cudaEventDestroy(e);
+  for (cudaEvent_t e : cmp_ev) cudaEventDestroy(e);
+  if (h2d_stream) cudaStreamDestroy(h2d_stream);
+  if (d2h_stream) cudaStreamDestroy(d2h_stream);
   if (h_in_dev) cudaFree(h_in_dev);
   if (h_out_dev) cudaFree(h_out_dev);
   if (h_ws_dev) cudaFree(h_ws_dev);
@@ -814,6 +820,105 @@ static int run_group(const std::vector<stencil_plan_s*>& Ps, const std::vector<c
     for (size_t k = 0; k < np; ++k) src[k] = dst[k];
   }
   SM_CUDA(cudaGetLastError());
+  return STENCIL_OK;
+}
+
+// End to end with host buffers, pipelined over z-chunks (views with enough
+// planes, no slab). Chunk k's input planes [Z_{k-1}, Z_k) go up on a copy
+// stream; then, on the plan's stream, launch i of the time loop (fusing up to
+// T steps) computes the planes it can now reach, [Z_{k-1} - sk_i, Z_k - sk_i)
+// with the skew sk_i = (i+1)*T*E (E = max z extent; the first chunk starts at
+// 0, the last runs to the top) -- a time-skewed wavefront that computes every
+// (launch, plane) exactly once -- and the planes that became final,
+// [Z_{k-1} - sk_last, Z_k - sk_last), go down on a second copy stream. The
+// H2D of chunk k+1, the sweep of chunk k and the D2H of chunk k-1 overlap
+// (PCIe is full duplex) instead of running back to back.
+// Correctness: launch i reads the buffer of launch i-1 on
+// [lo - t_i*zlo, hi + t_i*zhi); its top is <= Z_k - sk_{i-1}, already computed;
+// its bottom is >= Z_{k-1} - sk_i - T*E = Z_{k-1} - sk_{i+1}, at or above
+// everything an earlier chunk's launch i+1 wrote into that same-parity buffer,
+// so nothing it needs was overwritten; final planes below Z_k - sk_last are
+// never written again (later chunks write above Z_k - sk_i >= Z_k - sk_last);
+// frame points are time-invariant. Same kernels and per-point order as
+// stencil_run: bitwise equal results. *done = false: the plan does not qualify.
+static int run_host_pipelined(stencil_plan_s* P, const void* hin, void* hout, int steps, bool* done) {
+  *done = false;
+  const int nz = (int)P->vdims[0];
+  const int E = std::max(P->pat.zlo, P->pat.zhi);
+  if (P->comm || steps < 1 || P->timing || nz < 64) return STENCIL_OK;
+  const int K = std::min(16, nz / 32);   // chunks of >= 32 planes; more chunks = shorter fill and drain
+  const int T = P->var.family == FAM_TILED || P->var.family == FAM_STREAM_TB ? P->var.tt : 1;
+  const int launches = (steps + T - 1) / T;
+  const long long skew = (long long)launches * T * E;
+  if (K < 2 || skew * 2 >= nz / K) return STENCIL_OK;   // the skew must stay well inside a chunk
+  SM_TRY(ensure_loaded(P));
+  const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+  const size_t pb = (size_t)P->vdims[1] * P->vdims[2] * elem;
+  char* din = (char*)P->h_in_dev;
+  char* dout = (char*)P->h_out_dev;
+  char* dws = (char*)P->ws;
+  if (!P->h2d_stream) SM_CUDA(cudaStreamCreateWithFlags(&P->h2d_stream, cudaStreamNonBlocking));
+  if (!P->d2h_stream) SM_CUDA(cudaStreamCreateWithFlags(&P->d2h_stream, cudaStreamNonBlocking));
+  while ((int)P->h2d_ev.size() < K) {
+    cudaEvent_t a, b;
+    SM_CUDA(cudaEventCreateWithFlags(&a, cudaEventDisableTiming));
+    SM_CUDA(cudaEventCreateWithFlags(&b, cudaEventDisableTiming));
+    P->h2d_ev.push_back(a);
+    P->cmp_ev.push_back(b);
+  }
+  // the copy streams start after everything queued on the plan's stream
+  SM_CUDA(cudaEventRecord(P->cmp_ev[0], P->stream));
+  SM_CUDA(cudaStreamWaitEvent(P->h2d_stream, P->cmp_ev[0], 0));
+  SM_CUDA(cudaStreamWaitEvent(P->d2h_stream, P->cmp_ev[0], 0));
+  const GridArg g = make_grid(P, P->var.vx);
+  std::vector<Variant> vs(launches);
+  std::vector<Kernel> ks(launches);
+  for (int i = 0; i < launches; ++i) {
+    const int tl = std::min(T, steps - i * T);
+    if (tl == T) { vs[i] = P->var; ks[i] = P->kern; }
+    else SM_TRY(get_tb_rem_kernel(P, tl, &vs[i], &ks[i]));
+  }
+  int d_done = 0;   // planes already sent down
+  for (int k = 0; k < K; ++k) {
+    const int z0 = (int)((long long)nz * k / K), z1 = (int)((long long)nz * (k + 1) / K);
+    SM_CUDA(cudaMemcpyAsync(din + z0 * pb, (const char*)hin + z0 * pb, (z1 - z0) * pb, cudaMemcpyHostToDevice,
+                            P->h2d_stream));
+    SM_CUDA(cudaEventRecord(P->h2d_ev[k], P->h2d_stream));
+    SM_CUDA(cudaStreamWaitEvent(P->stream, P->h2d_ev[k], 0));
+    // a4 for these planes: the frame into every buffer the sweep writes
+    GridArg gf = g;
+    gf.nz = z1 - z0;
+    gf.uz0 = std::min(std::max(g.uz0 - z0, 0), gf.nz);
+    gf.uz1 = std::min(std::max(g.uz1 - z0, gf.uz0), gf.nz);
+    SM_TRY(launch_frame_copy(din + z0 * pb, dout + z0 * pb, elem, gf, P->stream));
+    if (launches >= 2) SM_TRY(launch_frame_copy(din + z0 * pb, dws + z0 * pb, elem, gf, P->stream));
+    const void* src = din;
+    for (int i = 0; i < launches; ++i) {
+      const int sk = (i + 1) * T * E;
+      char* dst = ((launches - 1 - i) % 2 == 0) ? dout : dws;
+      const int lo = std::max(g.cz0, k == 0 ? 0 : z0 - sk);
+      const int hi = std::min(g.cz1, k == K - 1 ? nz : z1 - sk);
+      if (hi > lo) {
+        GridArg gl = g;
+        gl.cz0 = lo;
+        gl.cz1 = hi;
+        SM_TRY(launch_sweep(P, vs[i], ks[i], src, dst, gl));
+      }
+      src = dst;
+    }
+    SM_CUDA(cudaEventRecord(P->cmp_ev[k], P->stream));
+    const int d1 = k == K - 1 ? nz : std::max(d_done, (int)(z1 - skew));
+    if (d1 > d_done) {
+      SM_CUDA(cudaStreamWaitEvent(P->d2h_stream, P->cmp_ev[k], 0));
+      SM_CUDA(cudaMemcpyAsync((char*)hout + d_done * pb, dout + d_done * pb, (d1 - d_done) * pb,
+                              cudaMemcpyDeviceToHost, P->d2h_stream));
+      d_done = d1;
+    }
+  }
+  SM_CUDA(cudaGetLastError());
+  SM_CUDA(cudaStreamSynchronize(P->d2h_stream));
+  SM_CUDA(cudaStreamSynchronize(P->stream));
+  *done = true;
   return STENCIL_OK;
 }
 
@@ -1072,6 +1177,16 @@ int stencil_run_host(stencil_plan_t P, const void* in_host, void* out_host, int 
     if (!P->h_ws_dev) SM_CUDA(cudaMalloc(&P->h_ws_dev, bytes));
     P->ws = P->h_ws_dev;
     P->ws_bytes = bytes;
+  }
+  {
+    bool done = false;
+    const char* np = getenv("STENCIL_NO_PIPELINE");   // dev override: unpipelined path
+    const int rc = (np && atoi(np)) ? STENCIL_OK : run_host_pipelined(P, in_host, out_host, steps, &done);
+    if (rc != STENCIL_OK || done) {
+      P->ws = saved_ws;
+      P->ws_bytes = saved_b;
+      return rc;
+    }
   }
   SM_CUDA(cudaMemcpyAsync(P->h_in_dev, in_host, bytes, cudaMemcpyHostToDevice, P->stream));
   int rc = run_device(P, P->h_in_dev, P->h_out_dev, steps);

@@ -201,6 +201,8 @@ struct stencil_plan_s {
   void* h_in_dev = nullptr;
   void* h_out_dev = nullptr;
   void* h_ws_dev = nullptr;
+  cudaStream_t h2d_stream = nullptr, d2h_stream = nullptr;   // pipelined stencil_run_host
+  std::vector<cudaEvent_t> h2d_ev, cmp_ev;
 
   // rows of the last OC sweep (stencil_sweep_rows)
   std::vector<stencil_sweep_row_t> sweep_rows;

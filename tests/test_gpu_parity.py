@@ -8,6 +8,8 @@ bitwise equal to each other (canonical FMA order); integer outputs
 import concurrent.futures as cf
 import math
 
+import os
+
 import numpy as np
 import pytest
 
@@ -176,6 +178,38 @@ def test_run_host_end_to_end(gpu):
     p.run_host(np.ascontiguousarray(u0), out, 3)
     ref = oracle.sweep(u0, acc, c, 3, dtype="f32")
     assert _relerr(out, ref) <= 1e-5
+
+
+@pytest.mark.parametrize("name,dims,dtype,oc,prm,steps", [
+    ("heat3d", (160, 40, 72), "f64", "ST_TB_BM_RT_PR", None, 5),      # TB with a remainder launch
+    ("heat3d", (130, 33, 64), "f64", "base", None, 4),
+    ("random3d:2:5", (150, 36, 48), "f64", "ST_BM_RT_PR", None, 3),
+    ("random3d:1:0", (140, 40, 80), "f64", "ST_TB_CM_RT", {"merge": 2}, 6),
+    ("star25", (200, 30, 72), "f32", "ST_RT_PR", None, 2),
+    ("box125", (128, 26, 40), "f64", "TB_BM", {"tb_steps": 2}, 3),
+    ("random2d:3:8", (700, 90), "f64", "ST_BM_RT_PR", None, 4)])
+def test_run_host_pipelined(gpu, name, dims, dtype, oc, prm, steps):
+    """stencil_run_host pipelines H2D / sweep / D2H over z-chunks with a
+    time-skewed wavefront (api.cpp run_host_pipelined): bitwise equal to the
+    device-buffer run and to the unpipelined host path, and within tolerance
+    of the oracle."""
+    torch = _torch()
+    acc, c = si.config_stencil(name)
+    u0 = np.ascontiguousarray(si.make_field(dims, 17, dtype))
+    p = sm.Plan(dims, acc, c, dtype, sm.oc_from_name(oc), prm)
+    out = np.empty_like(u0)
+    p.run_host(u0, out, steps)
+    dev = _run(p, u0, dtype, steps)
+    assert np.array_equal(out, dev)
+    os.environ["STENCIL_NO_PIPELINE"] = "1"
+    try:
+        out2 = np.empty_like(u0)
+        sm.Plan(dims, acc, c, dtype, sm.oc_from_name(oc), prm).run_host(u0, out2, steps)
+    finally:
+        del os.environ["STENCIL_NO_PIPELINE"]
+    assert np.array_equal(out, out2)
+    ref = oracle.sweep(u0, acc, c, steps, dtype=dtype)
+    assert _relerr(out, ref) <= TOL[dtype]
 
 
 def test_oc_sweep_label(gpu):
