@@ -111,7 +111,7 @@ class ClockSampler:
                         self.reasons.add(k)
             except Exception:
                 pass
-            self._stop.wait(0.005)
+            self._stop.wait(0.02)
 
     def __enter__(self):
         if self.nv:

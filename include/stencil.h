@@ -168,9 +168,14 @@ int stencil_plan_info(stencil_plan_t plan, stencil_plan_info_t *info);
  * TB OCs launch ceil(steps/T) times, the last launch fusing the remainder. */
 int stencil_run(stencil_plan_t plan, const void *in_dev, void *out_dev, int steps);
 
-/* End-to-end form: `in_host` / `out_host` are host buffers of the grid. The
- * call copies in_host to device buffers it owns, runs `steps` steps with the
- * plan's OC, copies the result back and synchronises the plan's stream. */
+/* End-to-end form: `in_host` / `out_host` are host buffers of the grid (pinned
+ * memory for full PCIe speed). The call copies in_host to device buffers it
+ * owns, runs `steps` steps with the plan's OC, copies the result back and
+ * returns when out_host holds it (the plan's stream is synchronised). Single-GPU
+ * plans whose slowest view axis has >= 64 planes are pipelined over z-chunks:
+ * the upload of chunk k+1, a time-skewed sweep of chunk k and the download of
+ * chunk k-1 overlap on two internal copy streams; the result is bitwise that of
+ * stencil_run. Errors as stencil_run. */
 int stencil_run_host(stencil_plan_t plan, const void *in_host, void *out_host, int steps);
 
 /* The label generator: for each of the 30 OCs in ascending id

@@ -846,11 +846,13 @@ static int run_host_pipelined(stencil_plan_s* P, const void* hin, void* hout, in
   const int nz = (int)P->vdims[0];
   const int E = std::max(P->pat.zlo, P->pat.zhi);
   if (P->comm || steps < 1 || P->timing || nz < 64) return STENCIL_OK;
-  const int K = std::min(16, nz / 32);   // chunks of >= 32 planes; more chunks = shorter fill and drain
   const int T = P->var.family == FAM_TILED || P->var.family == FAM_STREAM_TB ? P->var.tt : 1;
   const int launches = (steps + T - 1) / T;
   const long long skew = (long long)launches * T * E;
-  if (K < 2 || skew * 2 >= nz / K) return STENCIL_OK;   // the skew must stay well inside a chunk
+  // up to 16 chunks (shorter fill and drain) of >= 32 planes and more than
+  // twice the skew (the wavefront must stay well inside a chunk)
+  const int K = (int)std::min<long long>(16, nz / std::max<long long>(32, 2 * skew + 1));
+  if (K < 2) return STENCIL_OK;
   SM_TRY(ensure_loaded(P));
   const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
   const size_t pb = (size_t)P->vdims[1] * P->vdims[2] * elem;

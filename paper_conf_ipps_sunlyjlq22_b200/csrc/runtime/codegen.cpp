@@ -349,7 +349,12 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   }
   o << "};\n";
   const char* T = f32 ? "float" : "double";
-  o << "__device__ constexpr " << T << " g_coef[" << pat.nnz << "] = {";
+  // (tried: fp64 coefficients in __constant__ memory instead of immediates --
+  // ptxas then stages them through uniform registers with LDCU + R2UR and the
+  // order-2 random kernel grew from 86 to 132 registers; the UMOV-materialised
+  // immediates stay)
+  const bool cbank = false;
+  o << (cbank ? "__constant__ " : "__device__ constexpr ") << T << " g_coef[" << pat.nnz << "] = {";
   for (int i = 0; i < pat.nnz; ++i) o << hexfloat(pat.c[i], f32) << (i + 1 < pat.nnz ? "," : "");
   o << "};\n";
   // Packed FFMA2 pairs for fp32 are off by default: measured on C3 (star25,
@@ -389,7 +394,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
     << ", YLO = " << pat.ylo << ", YHI = " << pat.yhi << ", XLO = " << pat.xlo << ", XHI = " << pat.xhi
     << ", NZ = " << NZ << ", NY = " << NY << ", NX = " << NX << ";\n";
   o << "  static __device__ __forceinline__ constexpr int idx(int z, int y, int x) { return g_idx[z][y][x]; }\n";
-  o << "  static __device__ __forceinline__ constexpr T coef(int i) { return g_coef[i]; }\n";
+  o << "  static __device__ __forceinline__ " << (cbank ? "" : "constexpr ") << "T coef(int i) { return g_coef[i]; }\n";
   o << "  static constexpr int NOPS = " << ops.size() << ";\n";
   // retiming queue rotation: NZ unrolled plane bodies while they stay small,
   // register shifts beyond. Measured (B200, 512^3 / 768^3): the unrolled form
