@@ -110,6 +110,7 @@ typedef struct {
     int32_t reg_split[2];     /* warp-specialised ST_TB_RT kernel: registers per thread of the
                                  producer/intermediate-stage warps and of the last-stage warps
                                  after setmaxnreg (0, 0 = no split) */
+    int32_t xshift;           /* ST_TB_RT kernel uses the aligned-window ring geometry (§6.1) */
 } stencil_plan_info_t;
 
 /* ---------------------------------------------------------------------------

@@ -1118,6 +1118,7 @@ int stencil_plan_info(stencil_plan_t P, stencil_plan_info_t* info) {
   snprintf(info->kernel_name, sizeof info->kernel_name, "%s", P->lowered.c_str());
   info->reg_split[0] = P->var.reg_lo;
   info->reg_split[1] = P->var.reg_hi;
+  info->xshift = P->var.xshift ? 1 : 0;
   return STENCIL_OK;
 }
 

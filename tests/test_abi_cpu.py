@@ -179,3 +179,19 @@ def test_tbrt_register_split_choice():
     assert q.info["reg_split"] == (0, 0)
     r = _plan((512, 512, 512), acc, c, "f64", sm.oc_from_name("ST_BM_RT_PR"))
     assert r.info["reg_split"] == (0, 0)            # only the TB-RT family splits
+
+
+def test_tbrt_aligned_window_choice():
+    """The aligned-window ring geometry is taken only where the
+    shifted TMA box start stays 16-byte aligned (T*XLO a multiple of 16 B) and
+    the window loads drop by >= 15%: fp64 order-1 Algorithm-1 stencils (full
+    3x3 in-plane rows) take it, the heat star (9% fewer loads) does not, and
+    fp32 heat (T*XLO = 2 floats = 8 B: a misaligned box start) must not."""
+    prm = {"bx": 64, "by": 8, "vx": 2, "merge": 4, "tb_steps": 2, "pr_stages": 3}
+    oc = sm.oc_from_name("ST_TB_BM_RT_PR")
+    acc, c = si.config_stencil("random3d:1:0")
+    assert _plan((64, 64, 64), acc, c, "f64", oc, prm).info["xshift"]
+    acc, c = si.config_stencil("heat3d")
+    assert not _plan((64, 64, 64), acc, c, "f64", oc, prm).info["xshift"]
+    assert not _plan((64, 64, 64), acc, c, "f32", oc).info["xshift"]
+    assert not _plan((64, 64, 64), acc, c, "f64", sm.oc_from_name("ST_BM_RT_PR")).info["xshift"]
