@@ -1017,6 +1017,14 @@ int stencil_plan_create(stencil_plan_t* plan, int ndim, const int64_t* dims, int
   // Default tiles shrink until the shared-memory footprint fits (high-order
   // stencils under TB need smaller tiles); user-given fields are kept.
   const bool user_bz = params && params->bz, user_by = params && params->by, user_bx = params && params->bx;
+  // single-step 3-D streaming of an HBM-bound stencil with a tall y extent:
+  // taller tiles, the 2*r halo rows each tile re-reads per plane would otherwise be
+  // 2x its own rows (measured on C3, star25 r = 4, 768^3 fp32: ST_BM_RT_PR 454 ->
+  // 600 GStencil/s, ST_CM_RT_PR 435 -> 614). FMA-bound stencils (>= 48 FMAs per
+  // point) keep by 2: order-4 random 1024^3 fp64 54.2 (by 2) vs 50.1 (by 4).
+  if (!user_by && ndim == 3 && family_of(oc, P->params.smem) == FAM_STREAM &&
+      P->pat.ylo + P->pat.yhi >= 6 && P->pat.nnz < 48 && P->params.by < 4)
+    P->params.by = 4;
   if (!user_bx && family_of(oc, P->params.smem) != FAM_NAIVE) {
     // keep the default halo tile within one TMA box (<= 256 elements per row)
     const int elem = dtype == STENCIL_F64 ? 8 : 4;
