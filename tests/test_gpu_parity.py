@@ -230,9 +230,12 @@ def test_oc_sweep_label(gpu):
 
 
 @pytest.mark.parametrize("cfg,ocs,stencil", [
-    ("C2", ["ST_RT_PR", "ST_PR", "base", "ST_TB_BM_RT_PR"], None), ("C3", ["ST_RT_PR", "ST_BM_RT_PR"], None),
-    ("C4", ["ST_RT_PR", "TB"], None), ("C5", ["ST_BM_RT_PR"], "random3d:4:12"),
-    ("C5", ["ST_TB_BM_RT_PR"], "random3d:1:0"), ("N2", ["TB_BM", "ST_BM_RT_PR"], "random2d:3:8")])
+    ("C2", ["ST_RT_PR", "ST_PR", "base", "ST_TB_BM_RT_PR"], None),
+    ("C3", ["ST_RT_PR", "ST_BM_RT_PR", "ST_CM_RT_PR"], None),
+    ("C4", ["ST_RT_PR", "TB", "ST_CM_RT_PR"], None), ("C5", ["ST_BM_RT_PR"], "random3d:4:12"),
+    ("C5", ["ST_TB_BM_RT_PR"], "random3d:1:0"), ("C5", ["ST_BM_RT_PR", "ST_CM_RT_PR"], "random3d:2:4"),
+    ("N2", ["TB_BM", "ST_BM_RT_PR"], "random2d:3:8"), ("N2", ["TB_BM"], "random2d:1:0"),
+    ("N2", ["ST_RT_PR", "TB_BM"], "random2d:4:12")])
 def test_full_size_sampled(gpu, cfg, ocs, stencil):
     """BASELINE sizes, the bench's launch configuration (default settings of
     the OCs the bench labels), sampled points vs the oracle on their
