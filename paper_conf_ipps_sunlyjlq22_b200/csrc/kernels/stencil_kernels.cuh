@@ -220,6 +220,24 @@ struct SmemPlane {                    // shared memory, compile-time row pitch
   }
 };
 
+// Even/odd-split rows (k_stream_tb_rt, S::SPLITMID; fp64, VX = 2): column c of
+// a row lives at (c & 1) * LX/2 + (c >> 1). A thread's x-neighbour columns then
+// come from contiguous 8-byte loads (the odd array for c - 1, the even one for
+// c + 2) instead of 8-byte halves of 16-byte vectors at a 16-byte stride, which
+// cost a 16-byte vector's shared-memory wavefronts for half the data.
+template <class T, int LX>
+struct SplitPlane {
+  const T* p;                          // even array of row 0 at the thread's first output vector
+  __device__ __forceinline__ void get(int j, int kv, T (&w)[2]) const {
+    w[0] = p[j * LX + kv];
+    w[1] = p[j * LX + LX / 2 + kv];
+  }
+};
+template <int LX>
+__device__ __forceinline__ int split_idx(int row, int col) {
+  return row * LX + (col & 1) * (LX / 2) + (col >> 1);
+}
+
 template <class T, int VX, int NROW>
 struct GlobalPlane {                  // global memory through the read-only path
   const T* p;                          // element (plane z+dz, col 0) -- rows via rowoff
@@ -1132,7 +1150,8 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     const int gx0 = xb - G::TXL + (t % G::NTX) * VX;
     const int gy0 = yb - G::HY0 + (t / G::NTX) * MI;
     const int lb_r = (gy0 - Y0) * C::LX + (gx0 - xb + XO_R);   // tile origin in the source ring
-    const int lb = (gy0 - Y0) * C::LX + (gx0 - xb + XO_W);     // ... in the stage's own ring
+    const int lrow = gy0 - Y0, lcol = gx0 - xb + XO_W;
+    const int lb = lrow * C::LX + lcol;                         // ... in the stage's own ring
     const int ry1 = yb + BY * M + G::HY1;
     // rows: bit m = writable (inside R_s rows and the array), bit 8+m = inside the update box
     unsigned rows = 0, allup = 1;
@@ -1179,17 +1198,26 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         const bool zin = zo >= 0 && zo < g.nz;
         const bool zupd = zo >= g.uz0 && zo < g.uz1;
         const T(&res)[MI][VX] = acc[(U + 1) % NZ];
+        constexpr bool SPL = S::SPLITMID && s == TT - 1;  // the ring the last stage reads
         if (zupd && fast) {                              // interior: vector stores (don't-care
 #pragma unroll                                          // values past R_s stay in the buffer)
           for (int m = 0; m < MI; ++m)
-            if (rows & (1u << m)) stg_vec<T, VX>(dst + lb + m * C::LX, res[m]);
+            if (rows & (1u << m)) {
+              if constexpr (SPL) {
+                T* d = dst + split_idx<C::LX>(lrow + m, lcol);
+                d[0] = res[m][0];
+                d[C::LX / 2] = res[m][1];
+              } else {
+                stg_vec<T, VX>(dst + lb + m * C::LX, res[m]);
+              }
+            }
         } else if (zin && act) {                         // frame / edge tiles
 #pragma unroll
           for (int m = 0; m < MI; ++m) {
             if (!(rows & (1u << m))) continue;
             const bool rowupd = zupd && (rows & (1u << (8 + m)));
             T* d = dst + lb + m * C::LX;
-            if (rowupd && xfast) {
+            if (rowupd && xfast && !SPL) {
               stg_vec<T, VX>(d, res[m]);
             } else {
               const T* frame = in + (i64)zo * g.sz + (i64)(gy0 + m) * g.sy;
@@ -1198,7 +1226,9 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
                 const int gx = gx0 + v;
                 if (gx < 0 || gx >= g.nx || gx - xb + XO_W >= C::LX) continue;
                 const bool upd = rowupd && gx >= g.ux0 && gx < g.ux1;
-                d[v] = upd ? res[m][v] : (s == 1 ? fr[m * C::LX + v] : __ldg(frame + gx));
+                const T val = upd ? res[m][v] : (s == 1 ? fr[m * C::LX + v] : __ldg(frame + gx));
+                if constexpr (SPL) dst[split_idx<C::LX>(lrow + m, lcol + v)] = val;
+                else d[v] = val;
               }
             }
           }
@@ -1237,8 +1267,14 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         mbar_wait_sleep(&fin[si], (unsigned)((j / MR) & 1));
         if constexpr (!S::RTSHIFT) zero_acc<T, VX, M>(acc[U]);
         if (act) {
-          SmemPlane<T, VX, C::LX> pl{mid + (MR * (TT - 2) + si) * C::PLANE + row0 * C::LX + col0};
-          run_scatter<S, VX, M, U>(pl, acc);
+          const T* pm = mid + (MR * (TT - 2) + si) * C::PLANE;
+          if constexpr (S::SPLITMID) {
+            SplitPlane<T, C::LX> pl{pm + row0 * C::LX + (col0 >> 1)};
+            run_scatter<S, VX, M, U>(pl, acc);
+          } else {
+            SmemPlane<T, VX, C::LX> pl{pm + row0 * C::LX + col0};
+            run_scatter<S, VX, M, U>(pl, acc);
+          }
         }
         mbar_arrive(&ein[si]);
         const int z = pin0 + j - TT * S::ZHI;

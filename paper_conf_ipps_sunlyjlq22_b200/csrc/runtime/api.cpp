@@ -321,6 +321,9 @@ static int resolve_variant(stencil_plan_s* P) {
       v.xshift = l1 <= 0.85 * l0;
     }
     if (const char* nx = getenv("STENCIL_XSHIFT")) v.xshift = tma_ok && atoi(nx) != 0;   // dev override
+    // even/odd-split last intermediate ring (fp64, 16-byte vectors of 2, rounded geometry)
+    v.splitmid = elem == 8 && v.vx == 2 && !v.xshift;
+    if (const char* sp = getenv("STENCIL_SPLITMID")) v.splitmid = v.splitmid && atoi(sp) != 0;   // dev override
     choose_regsplit(&v, P->pat, elem);
     v.ws_threads = v.tbrt_threads(P->pat, elem);
   }

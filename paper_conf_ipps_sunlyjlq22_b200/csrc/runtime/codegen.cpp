@@ -384,6 +384,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   if (const char* e = getenv("STENCIL_MINB")) minb = atoi(e);   // dev override
   o << "  static constexpr int MINB = " << minb << ";\n";
   o << "  static constexpr int MIDR = " << v.mid_slots() << ";\n";
+  o << "  static constexpr bool SPLITMID = " << (v.splitmid ? "true" : "false") << ";\n";
   o << "  static constexpr bool XSHIFT = " << (v.xshift ? "true" : "false") << ";\n";
   o << "  static constexpr int XSH = " << (v.xshift ? pat.xlo % std::max(v.vx, 1) : 0) << ";\n";
   o << "  static constexpr int REG_LO = " << v.reg_lo << ", REG_HI = " << v.reg_hi << ";\n";

@@ -86,6 +86,7 @@ struct Variant {
   long long sy = 0, sz = 0;   // row / plane strides baked into the kernel (0 = run time)
   int reg_lo = 0, reg_hi = 0; // k_stream_tb_rt register split (setmaxnreg; 0 = off)
   bool xshift = false;        // k_stream_tb_rt: per-step ring geometry with aligned windows
+  bool splitmid = false;      // k_stream_tb_rt: even/odd-split rows in the last intermediate ring
   std::string name_expr(const char* desc) const;
   int threads() const;
   int smem_bytes(const Pattern& p, int elem) const;
