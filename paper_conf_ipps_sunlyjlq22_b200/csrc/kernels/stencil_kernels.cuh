@@ -1009,8 +1009,12 @@ struct TbRtStage {
   static constexpr int HX0 = (TT - s) * S::XLO, HX1 = (TT - s) * S::XHI;
   static constexpr int HY0 = (TT - s) * S::YLO, HY1 = (TT - s) * S::YHI;
   // tile x origin = xb - TXL (S::XSHIFT: exactly the region's left edge, see StreamTbRtCfg)
-  static constexpr int TXL = S::XSHIFT ? HX0 : ((HX0 + VX - 1) / VX) * VX;
-  static constexpr int NTX = (TXL + BX + HX1 + VX - 1) / VX;
+  // intermediate steps use thread tiles of S::MVX x MI (S::MVX = 1: scalar
+  // columns, so every shared-memory access of the stage is a contiguous 8-byte
+  // warp access instead of 16-byte vectors with half-used neighbours)
+  static constexpr int VXM = S::MVX;
+  static constexpr int TXL = S::XSHIFT ? HX0 : ((HX0 + VXM - 1) / VXM) * VXM;
+  static constexpr int NTX = (TXL + BX + HX1 + VXM - 1) / VXM;
   static constexpr int RY = BY * M + HY0 + HY1;
   static constexpr int NTY = (RY + MI - 1) / MI;
   static constexpr int NT = NTX * NTY;
@@ -1144,10 +1148,11 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     if (done || warp < W0 || warp >= W0 + G::W) return;
     done = true;
     constexpr int XO_R = C::xoff(s - 1), XO_W = C::xoff(s);   // source / own ring geometry
-    constexpr bool XOVER = XO_W - G::TXL + G::NTX * VX > C::LX;
+    constexpr int MV = G::VXM;
+    constexpr bool XOVER = XO_W - G::TXL + G::NTX * MV > C::LX;
     const int t = tid - 32 * W0;
     const bool act = t < G::NT;
-    const int gx0 = xb - G::TXL + (t % G::NTX) * VX;
+    const int gx0 = xb - G::TXL + (t % G::NTX) * MV;
     const int gy0 = yb - G::HY0 + (t / G::NTX) * MI;
     const int lb_r = (gy0 - Y0) * C::LX + (gx0 - xb + XO_R);   // tile origin in the source ring
     const int lrow = gy0 - Y0, lcol = gx0 - xb + XO_W;
@@ -1163,14 +1168,14 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
       rows |= (wr ? 1u << m : 0u) | (up ? 1u << (8 + m) : 0u);
       allup &= (gy >= ry1 || up) ? 1u : 0u;
     }
-    const bool xfast = gx0 >= g.ux0 && gx0 + VX <= g.ux1 && (!XOVER || gx0 - xb + XO_W + VX <= C::LX);
+    const bool xfast = gx0 >= g.ux0 && gx0 + MV <= g.ux1 && (!XOVER || gx0 - xb + XO_W + MV <= C::LX);
     const bool fast = act && xfast && allup;
     unsigned long long* fin = s == 1 ? full_in : full_s(s - 1);
     unsigned long long* ein = s == 1 ? empty_in : empty_s(s - 1);
     constexpr int DIN = s == 1 ? NR : MR;
-    T acc[NZ][MI][VX];
+    T acc[NZ][MI][MV];
 #pragma unroll
-    for (int q = 0; q < NZ; ++q) zero_acc<T, VX, MI>(acc[q]);
+    for (int q = 0; q < NZ; ++q) zero_acc<T, MV, MI>(acc[q]);
     // NZ unrolled plane bodies (compile-time queue rotation), or one body and
     // a register shift of the queue for large op tables (S::RTSHIFT)
     constexpr int UNR = S::RTSHIFT ? 1 : NZ;
@@ -1183,10 +1188,10 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         const int si = j % DIN;
         const T* src = s == 1 ? ring0 + si * C::PLANE : mid + (MR * (s - 2) + si) * C::PLANE;
         mbar_wait_sleep(&fin[si], (unsigned)((j / DIN) & 1));
-        if constexpr (!S::RTSHIFT) zero_acc<T, VX, MI>(acc[U]);   // a new output plane starts
+        if constexpr (!S::RTSHIFT) zero_acc<T, MV, MI>(acc[U]);   // a new output plane starts
         if (act) {
-          SmemPlane<T, VX, C::LX> pl{src + lb_r - S::XSH};
-          run_scatter_ops<S, typename S::Mid, VX, MI, U>(pl, acc);
+          SmemPlane<T, MV, C::LX> pl{src + lb_r - S::XSH};
+          run_scatter_ops<S, typename S::Mid, MV, MI, U>(pl, acc);
         }
         if (s > 1) mbar_arrive(&ein[si]);                // input slot read (stage 1: below)
         const int so = j % MR;
@@ -1197,18 +1202,17 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         const T* fr = ring0 + ((j - S::ZHI + NR) % NR) * C::PLANE + lb_r;
         const bool zin = zo >= 0 && zo < g.nz;
         const bool zupd = zo >= g.uz0 && zo < g.uz1;
-        const T(&res)[MI][VX] = acc[(U + 1) % NZ];
+        const T(&res)[MI][MV] = acc[(U + 1) % NZ];
         constexpr bool SPL = S::SPLITMID && s == TT - 1;  // the ring the last stage reads
         if (zupd && fast) {                              // interior: vector stores (don't-care
 #pragma unroll                                          // values past R_s stay in the buffer)
           for (int m = 0; m < MI; ++m)
             if (rows & (1u << m)) {
               if constexpr (SPL) {
-                T* d = dst + split_idx<C::LX>(lrow + m, lcol);
-                d[0] = res[m][0];
-                d[C::LX / 2] = res[m][1];
+#pragma unroll
+                for (int v = 0; v < MV; ++v) dst[split_idx<C::LX>(lrow + m, lcol + v)] = res[m][v];
               } else {
-                stg_vec<T, VX>(dst + lb + m * C::LX, res[m]);
+                stg_vec<T, MV>(dst + lb + m * C::LX, res[m]);
               }
             }
         } else if (zin && act) {                         // frame / edge tiles
@@ -1218,11 +1222,11 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
             const bool rowupd = zupd && (rows & (1u << (8 + m)));
             T* d = dst + lb + m * C::LX;
             if (rowupd && xfast && !SPL) {
-              stg_vec<T, VX>(d, res[m]);
+              stg_vec<T, MV>(d, res[m]);
             } else {
               const T* frame = in + (i64)zo * g.sz + (i64)(gy0 + m) * g.sy;
 #pragma unroll
-              for (int v = 0; v < VX; ++v) {
+              for (int v = 0; v < MV; ++v) {
                 const int gx = gx0 + v;
                 if (gx < 0 || gx >= g.nx || gx - xb + XO_W >= C::LX) continue;
                 const bool upd = rowupd && gx >= g.ux0 && gx < g.ux1;
@@ -1235,7 +1239,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         }
         if (s == 1 && j >= S::ZHI) mbar_arrive(&ein[(j - S::ZHI) % NR]);   // frame source released
         mbar_arrive(&full_s(s)[so]);                     // stage-s plane written
-        if constexpr (S::RTSHIFT) shift_queue<T, NZ, MI, VX>(acc);
+        if constexpr (S::RTSHIFT) shift_queue<T, NZ, MI, MV>(acc);
       });
     }
   });

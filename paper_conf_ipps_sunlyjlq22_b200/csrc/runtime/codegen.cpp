@@ -138,7 +138,7 @@ int Variant::mid_rows(const Pattern& p, int elem) const {
   (void)p; (void)elem;
   if (family == FAM_STREAM_TB && rt)
     if (const char* e = getenv("STENCIL_MID_ROWS")) return atoi(e);   // dev override
-  return 2;
+  return midvx == 1 ? 4 : 2;   // scalar-column intermediate tiles: 1 x 4
 }
 
 // Slots of each intermediate-stage ring of k_stream_tb_rt (S::MIDR).
@@ -174,8 +174,9 @@ int Variant::tbrt_threads(const Pattern& p, int elem, int* wl_out) const {
   for (int s = 1; s < tt; ++s) {
     const int hx0 = (tt - s) * p.xlo, hx1 = (tt - s) * p.xhi;
     const int hy0 = (tt - s) * p.ylo, hy1 = (tt - s) * p.yhi;
-    const int txl = xshift ? hx0 : roundup(hx0, vx);
-    const int ntx = (txl + bx + hx1 + vx - 1) / vx;
+    const int mvx = midvx > 0 ? midvx : vx;
+    const int txl = xshift ? hx0 : roundup(hx0, mvx);
+    const int ntx = (txl + bx + hx1 + mvx - 1) / mvx;
     const int nty = (by * m + hy0 + hy1 + mi - 1) / mi;
     warps += (ntx * nty + 31) / 32;
   }
@@ -321,6 +322,7 @@ int count_window_loads(const Pattern& pat, int elem, const Variant& v) {
   for (uint32_t op : encode_ops(pat, v, false)) n += !(op >> 31);
   Variant vm = v;
   vm.family = FAM_STREAM; vm.cm = false; vm.m = v.mid_rows(pat, elem);
+  if (v.midvx > 0) vm.vx = v.midvx;
   for (uint32_t op : encode_ops(pat, vm, false)) n += !(op >> 31);
   return n;
 }
@@ -372,6 +374,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   if (v.family == FAM_STREAM_TB) {     // intermediate fused steps: VX x MI tiles, gather or (RT) scatter
     Variant vm = v;
     vm.family = FAM_STREAM; vm.cm = false; vm.m = mi;
+    if (v.midvx > 0) vm.vx = v.midvx;
     mops = encode_ops(pat, vm, pair);
   }
   o << "__device__ constexpr unsigned g_mops[" << std::max<size_t>(mops.size(), 1) << "] = {";
@@ -384,6 +387,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   if (const char* e = getenv("STENCIL_MINB")) minb = atoi(e);   // dev override
   o << "  static constexpr int MINB = " << minb << ";\n";
   o << "  static constexpr int MIDR = " << v.mid_slots() << ";\n";
+  o << "  static constexpr int MVX = " << (v.midvx > 0 ? v.midvx : std::max(v.vx, 1)) << ";\n";
   o << "  static constexpr bool SPLITMID = " << (v.splitmid ? "true" : "false") << ";\n";
   o << "  static constexpr bool XSHIFT = " << (v.xshift ? "true" : "false") << ";\n";
   o << "  static constexpr int XSH = " << (v.xshift ? pat.xlo % std::max(v.vx, 1) : 0) << ";\n";

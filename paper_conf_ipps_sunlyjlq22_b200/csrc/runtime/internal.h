@@ -87,6 +87,7 @@ struct Variant {
   int reg_lo = 0, reg_hi = 0; // k_stream_tb_rt register split (setmaxnreg; 0 = off)
   bool xshift = false;        // k_stream_tb_rt: per-step ring geometry with aligned windows
   bool splitmid = false;      // k_stream_tb_rt: even/odd-split rows in the last intermediate ring
+  int midvx = 0;              // k_stream_tb_rt: columns per thread of the intermediate steps (0 = vx)
   std::string name_expr(const char* desc) const;
   int threads() const;
   int smem_bytes(const Pattern& p, int elem) const;
