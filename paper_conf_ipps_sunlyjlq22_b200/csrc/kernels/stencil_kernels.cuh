@@ -530,16 +530,18 @@ k_tiled(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, G
     __syncthreads();
   }
 
-  // intermediate fused steps s = 1 .. TT-1 (temporal blocking)
+  // intermediate fused steps s = 1 .. TT-1 (temporal blocking); the step
+  // loop is unrolled at compile time so the region extents are constants (the
+  // point -> (x, y, z) decomposition is then multiply-shift, not runtime division)
   T* src = buf0;
   T* dst = buf1;
-#pragma unroll 1
-  for (int s = 1; s < TT; ++s) {
-    const int hz0 = (TT - s) * S::ZLO, hz1 = (TT - s) * S::ZHI;
-    const int hy0 = (TT - s) * S::YLO, hy1 = (TT - s) * S::YHI;
-    const int hx0 = (TT - s) * S::XLO, hx1 = (TT - s) * S::XHI;
-    const int RX = BX + hx0 + hx1, RY = BY * M + hy0 + hy1, RZ = BZ + hz0 + hz1;
-    const int n = RX * RY * RZ;
+  static_for<1, TT>([&](auto sc) {
+    constexpr int s = decltype(sc)::value;
+    constexpr int hz0 = (TT - s) * S::ZLO, hz1 = (TT - s) * S::ZHI;
+    constexpr int hy0 = (TT - s) * S::YLO, hy1 = (TT - s) * S::YHI;
+    constexpr int hx0 = (TT - s) * S::XLO, hx1 = (TT - s) * S::XHI;
+    constexpr int RX = BX + hx0 + hx1, RY = BY * M + hy0 + hy1, RZ = BZ + hz0 + hz1;
+    constexpr int n = RX * RY * RZ;
     for (int i = tid; i < n; i += C::THREADS) {
       const int rx = i % RX, ry = (i / RX) % RY, rz = i / (RX * RY);
       const int gx = xb - hx0 + rx, gy = yb - hy0 + ry, gz = zb - hz0 + rz;
@@ -563,7 +565,7 @@ k_tiled(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, G
     }
     __syncthreads();
     T* t = src; src = dst; dst = t;
-  }
+  });
 
   // final step: thread tile M x VX per plane, BZ planes
   const int tx = threadIdx.x, ty = threadIdx.y;
