@@ -481,7 +481,10 @@ struct TiledCfg {
   static constexpr int LZ = BZ + TT * (S::ZLO + S::ZHI);
   static constexpr int BUF = ((LX * LY * LZ * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
   static constexpr int NBUF = TT > 1 ? 2 : 1;
-  static constexpr int SMEM = NBUF * BUF * (int)sizeof(T) + 128;
+  // S::TMID > 0: intermediate steps in 1 x TMID register tiles (op table S::Mid,
+  // gather); the last tile of a column may read TMID - 1 rows past the buffer
+  static constexpr int PAD = (TT > 1 && S::TMID > 0) ? ((S::TMID * LX * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T) : 0;
+  static constexpr int SMEM = (NBUF * BUF + PAD) * (int)sizeof(T) + 128;
   static constexpr int THREADS = (BX / VX) * BY;
 };
 
@@ -494,7 +497,7 @@ k_tiled(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, G
   extern __shared__ __align__(128) unsigned char smem_raw[];
   T* buf0 = reinterpret_cast<T*>(smem_raw);
   T* buf1 = buf0 + C::BUF;
-  unsigned long long* bar = reinterpret_cast<unsigned long long*>(smem_raw + C::NBUF * C::BUF * sizeof(T));
+  unsigned long long* bar = reinterpret_cast<unsigned long long*>(smem_raw + (C::NBUF * C::BUF + C::PAD) * sizeof(T));
 
   const int tid = threadIdx.y * (BX / VX) + threadIdx.x;
   const int xa = (g.cx0 / C::ALN) * C::ALN;            // aligned x origin of the tile grid
@@ -541,6 +544,35 @@ k_tiled(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, G
     constexpr int hy0 = (TT - s) * S::YLO, hy1 = (TT - s) * S::YHI;
     constexpr int hx0 = (TT - s) * S::XLO, hx1 = (TT - s) * S::XHI;
     constexpr int RX = BX + hx0 + hx1, RY = BY * M + hy0 + hy1, RZ = BZ + hz0 + hz1;
+    if constexpr (S::TMID > 0) {
+      // 1 x MT register tiles: neighbouring lanes take neighbouring columns, so
+      // every shared-memory access is a contiguous warp access, and each loaded
+      // value feeds up to MT outputs of the column
+      constexpr int MT = S::TMID, NTY = (RY + MT - 1) / MT, NT = RX * NTY * RZ;
+      for (int t = tid; t < NT; t += C::THREADS) {
+        const int rx = t % RX, ty = (t / RX) % NTY, rz = t / (RX * NTY);
+        const int gx = xb - hx0 + rx, gy0 = yb - hy0 + ty * MT, gz = zb - hz0 + rz;
+        const int lb = ((gz - Z0) * C::LY + (gy0 - Y0)) * C::LX + (gx - X0);
+        T acc[MT][1];
+        zero_acc<T, 1, MT>(acc);
+        SmemPlane<T, 1, C::LX> pl[S::NZ];
+#pragma unroll
+        for (int zi = 0; zi < S::NZ; ++zi) pl[zi].p = src + lb + (zi - S::ZLO) * C::LY * C::LX;
+        run_gather_ops<S, typename S::Mid, 1, MT>(pl, acc);
+        const bool colok = gx >= 0 && gx < g.nx && gz >= 0 && gz < g.nz;
+        const bool colupd = gz >= g.uz0 && gz < g.uz1 && gx >= g.ux0 && gx < g.ux1;
+#pragma unroll
+        for (int m = 0; m < MT; ++m) {
+          const int gy = gy0 + m;
+          if (!colok || ty * MT + m >= RY || gy < 0 || gy >= g.ny) continue;
+          const int li = lb + m * C::LX;
+          dst[li] = (colupd && gy >= g.uy0 && gy < g.uy1) ? acc[m][0] : src[li];
+        }
+      }
+      __syncthreads();
+      T* t = src; src = dst; dst = t;
+      return;
+    }
     constexpr int n = RX * RY * RZ;
     for (int i = tid; i < n; i += C::THREADS) {
       const int rx = i % RX, ry = (i / RX) % RY, rz = i / (RX * RY);

@@ -339,6 +339,10 @@ static int resolve_variant(stencil_plan_s* P) {
     choose_regsplit(&v, P->pat, elem);
     v.ws_threads = v.tbrt_threads(P->pat, elem);
   }
+  if (fam == FAM_TILED && v.tt > 1) {
+    v.tiled_mid = 0;
+    if (const char* e = getenv("STENCIL_TILED_MID")) v.tiled_mid = std::max(0, std::min(8, atoi(e)));   // dev override
+  }
   const int thr = v.threads();
   if (thr < 32 || thr > 1024)
     SM_FAIL(STENCIL_E_OC_INFEASIBLE, "CTA of %d threads outside 32..1024", thr);

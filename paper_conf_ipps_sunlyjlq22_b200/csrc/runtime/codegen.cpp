@@ -196,7 +196,8 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     const int ly = by * m + tt * (p.ylo + p.yhi);
     const int lz = bz + tt * (p.zlo + p.zhi);
     const int buf = roundup(lx * ly * lz * elem, 128) / elem;
-    return (tt > 1 ? 2 : 1) * buf * elem + 128;
+    const int pad = tt > 1 && tiled_mid > 0 ? roundup(tiled_mid * lx * elem, 128) / elem : 0;   // TiledCfg::PAD
+    return ((tt > 1 ? 2 : 1) * buf + pad) * elem + 128;
   }
   if (family == FAM_STREAM) {
     const int xoff = roundup(p.xlo, aln);
@@ -371,6 +372,12 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   o << "};\n";
   std::vector<uint32_t> mops;
   const int mi = v.mid_rows(pat, f32 ? 4 : 8);
+  const int tmid = v.family == FAM_TILED && v.tt > 1 ? v.tiled_mid : 0;
+  if (tmid > 0) {                      // k_tiled intermediate steps: 1 x tmid tiles, gather
+    Variant vm = v;
+    vm.family = FAM_STREAM; vm.rt = false; vm.cm = false; vm.m = tmid; vm.vx = 1; vm.xshift = false;
+    mops = encode_ops(pat, vm, pair);
+  }
   if (v.family == FAM_STREAM_TB) {     // intermediate fused steps: VX x MI tiles, gather or (RT) scatter
     Variant vm = v;
     vm.family = FAM_STREAM; vm.cm = false; vm.m = mi;
@@ -387,6 +394,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   if (const char* e = getenv("STENCIL_MINB")) minb = atoi(e);   // dev override
   o << "  static constexpr int MINB = " << minb << ";\n";
   o << "  static constexpr int MIDR = " << v.mid_slots() << ";\n";
+  o << "  static constexpr int TMID = " << tmid << ";\n";
   o << "  static constexpr int MVX = " << (v.midvx > 0 ? v.midvx : std::max(v.vx, 1)) << ";\n";
   o << "  static constexpr bool SPLITMID = " << (v.splitmid ? "true" : "false") << ";\n";
   o << "  static constexpr bool XSHIFT = " << (v.xshift ? "true" : "false") << ";\n";

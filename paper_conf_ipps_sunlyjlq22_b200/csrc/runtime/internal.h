@@ -88,6 +88,7 @@ struct Variant {
   bool xshift = false;        // k_stream_tb_rt: per-step ring geometry with aligned windows
   bool splitmid = false;      // k_stream_tb_rt: even/odd-split rows in the last intermediate ring
   int midvx = 0;              // k_stream_tb_rt: columns per thread of the intermediate steps (0 = vx)
+  int tiled_mid = 0;          // k_tiled (TB): rows of the 1 x n intermediate-step register tiles (0 = scalar)
   std::string name_expr(const char* desc) const;
   int threads() const;
   int smem_bytes(const Pattern& p, int elem) const;
