@@ -340,7 +340,11 @@ static int resolve_variant(stencil_plan_s* P) {
     v.ws_threads = v.tbrt_threads(P->pat, elem);
   }
   if (fam == FAM_TILED && v.tt > 1) {
-    v.tiled_mid = 0;
+    // intermediate fused steps in 1 x 4 register tiles (k_tiled, S::TMID). Measured
+    // (same box, TB_BM / TB): N2 order-1 8192^2 582 -> 673 / 391 -> 439, order-2
+    // 423 -> 486, C2 heat 512^3 191 -> 240 / 138 -> 192 GStencil/s against one
+    // point per thread; 1 x 2 is within +-4%, 1 x 8 loses
+    v.tiled_mid = 4;
     if (const char* e = getenv("STENCIL_TILED_MID")) v.tiled_mid = std::max(0, std::min(8, atoi(e)));   // dev override
   }
   const int thr = v.threads();
