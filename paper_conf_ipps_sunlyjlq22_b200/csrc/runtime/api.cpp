@@ -124,9 +124,11 @@ static void default_params(uint32_t oc, int ndim, int dtype, stencil_params_t* p
     p->bx = 32; p->by = merge ? 4 : 8; p->bz = 1; p->vx = 1;
   } else if (fam == FAM_TILED) {
     p->vx = vmax; p->bx = 16 * vmax; p->by = merge ? 4 : 8; p->bz = (oc & STENCIL_OC_TB) ? 4 : 8;
-    // 2-D tiles merge 4 rows per thread (measured on N2's order-1 stencil, 8192^2
-    // fp64, TB_BM: merge 4 -> 597 GStencil/s, merge 2 -> 547)
-    if (ndim == 2) { p->bz = 1; if (merge) p->merge = 4; }
+    // 2-D tiles: 32 vectors wide, merge 4 rows per thread (measured on N2's
+    // order-1 stencil, 8192^2 fp64, TB_BM: merge 4 -> 597 GStencil/s, merge 2 -> 547;
+    // with register-tiled intermediate steps bx 64 -> 675, bx 32 -> 623; order 2:
+    // 487 vs 436)
+    if (ndim == 2) { p->bz = 1; p->bx = 32 * vmax; if (merge) p->merge = 4; }
   } else if (fam == FAM_STREAM) {
     // wide, shallow tiles: many small CTAs keep more TMA planes in flight per SM
     // (measured on C2: 128x2 fp64 tiles reach 92% of the copy bandwidth)
