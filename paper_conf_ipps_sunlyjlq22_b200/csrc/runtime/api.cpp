@@ -816,19 +816,37 @@ static int run_group(const std::vector<stencil_plan_s*>& Ps, const std::vector<c
                                P->stream));
       }
     } else if (slab && more) {
+      // The edge planes (the ones the neighbours need next) run on a
+      // high-priority stream concurrently with the interior: they start once
+      // the main stream has finished the previous launch (its interior read
+      // the planes they overwrite) and the previous exchange (main waited for
+      // it); the interior of this launch needs neither of them, and the next
+      // launch sees them through the exchange event.
       const int E = tl_next * std::max(P0->pat.zlo, P0->pat.zhi);
       for (size_t k = 0; k < np; ++k) {   // edge planes first
+        stencil_plan_s* P = Ps[k];
+        Comm* c = P->comm;
         GridArg g = gs[k];
         const int c0 = g.cz0, c1 = g.cz1;
+        cudaStream_t main_stream = P->stream;
+        const char* ser = getenv("STENCIL_EDGE_SERIAL");   // dev override: edges on the main stream
+        cudaStream_t es = (ser && atoi(ser)) ? main_stream : c->edge_stream;
+        SM_CUDA(cudaEventRecord(c->ev_main, main_stream));
+        SM_CUDA(cudaStreamWaitEvent(es, c->ev_main, 0));
+        P->stream = es;
+        int rc = STENCIL_OK;
         if (c1 - c0 > 2 * E) {
           g.cz1 = c0 + E;
-          SM_TRY(launch_sweep(Ps[k], vs[k], ks[k], src[k], dst[k], g));
+          rc = launch_sweep(P, vs[k], ks[k], src[k], dst[k], g);
           g.cz0 = c1 - E; g.cz1 = c1;
-          SM_TRY(launch_sweep(Ps[k], vs[k], ks[k], src[k], dst[k], g));
+          if (rc == STENCIL_OK) rc = launch_sweep(P, vs[k], ks[k], src[k], dst[k], g);
         } else {
-          SM_TRY(launch_sweep(Ps[k], vs[k], ks[k], src[k], dst[k], g));
+          rc = launch_sweep(P, vs[k], ks[k], src[k], dst[k], g);
         }
-        SM_CUDA(cudaEventRecord(Ps[k]->comm->ev_edge, Ps[k]->stream));
+        P->stream = main_stream;
+        if (rc != STENCIL_OK) return rc;
+        SM_CUDA(cudaEventRecord(c->ev_edge, es));
+        if (c1 - c0 <= 2 * E) SM_CUDA(cudaStreamWaitEvent(main_stream, c->ev_edge, 0));   // no interior
       }
       SM_TRY(exchange(Ps, dst, tl_next));
       for (size_t k = 0; k < np; ++k) {   // interior overlaps the exchange

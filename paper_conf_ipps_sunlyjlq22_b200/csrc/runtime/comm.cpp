@@ -20,6 +20,8 @@ void comm_destroy(Comm* c) {
   if (c->stream) cudaStreamDestroy(c->stream);
   if (c->ev_edge) cudaEventDestroy(c->ev_edge);
   if (c->ev_comm) cudaEventDestroy(c->ev_comm);
+  if (c->edge_stream) cudaStreamDestroy(c->edge_stream);
+  if (c->ev_main) cudaEventDestroy(c->ev_main);
   delete c;
 }
 
@@ -27,6 +29,10 @@ int comm_create_stream_events(Comm* c) {
   SM_CUDA(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
   SM_CUDA(cudaEventCreateWithFlags(&c->ev_edge, cudaEventDisableTiming));
   SM_CUDA(cudaEventCreateWithFlags(&c->ev_comm, cudaEventDisableTiming));
+  SM_CUDA(cudaEventCreateWithFlags(&c->ev_main, cudaEventDisableTiming));
+  int lo = 0, hi = 0;   // numerically lower = higher priority
+  SM_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+  SM_CUDA(cudaStreamCreateWithPriority(&c->edge_stream, cudaStreamNonBlocking, hi));
   return STENCIL_OK;
 }
 

@@ -147,6 +147,8 @@ struct Comm {
   cudaStream_t stream = nullptr;     // comm stream (owned per plan)
   cudaEvent_t ev_edge = nullptr;     // edge planes of dst written (main stream)
   cudaEvent_t ev_comm = nullptr;     // halo exchange into dst done (comm stream)
+  cudaStream_t edge_stream = nullptr;  // high-priority stream of the edge-plane kernels
+  cudaEvent_t ev_main = nullptr;     // main stream reached the edge launch (previous interior done)
   std::vector<stencil_plan_s*> peers;  // LOOPBACK: plans of all ranks (index = rank)
   const void* cur = nullptr;         // LOOPBACK: buffer this rank is exchanging (for peers)
   // P2P (fused halo): registered grids of this rank and its neighbours
