@@ -578,7 +578,13 @@ static int get_tb_rem_kernel(stencil_plan_s* P, int tt, Variant* vout, Kernel* k
   Variant v = P->var;
   v.tt = tt;
   v.reg_lo = v.reg_hi = 0;   // remainder launches are rare: no register split
-  if (tt < 2) v.xshift = false;
+  {
+    // the aligned-window geometry needs a 16-byte aligned TMA box start (tt * XLO
+    // elements); a remainder depth may not keep it (e.g. T = 4, remainder 3)
+    const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
+    const int aln = std::max(16 / elem, v.vx);
+    if (tt < 2 || (tt * P->pat.xlo) % aln != 0) v.xshift = false;
+  }
   if (v.family == FAM_STREAM_TB && tt == 1) v.family = FAM_STREAM;   // remainder of one step: plain ST
   const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
   if (v.family == FAM_STREAM_TB && v.rt) {

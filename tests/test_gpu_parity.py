@@ -296,6 +296,22 @@ def test_tb_rt_pipeline_settings(gpu, name, dims, dtype):
     assert ran >= 3
 
 
+def test_tb_rt_xshift_remainder(gpu):
+    """T = 4 aligned-window plan run for 7 steps: the remainder launch of depth 3
+    would start its TMA box 3 columns (24 bytes) left of the tile -- misaligned --
+    so it takes the rounded geometry; the result must still match."""
+    acc, c = si.config_stencil("random3d:1:0")
+    dims = (30, 50, 96)
+    u0 = si.make_field(dims, 41, "f64")
+    ref = oracle.sweep(u0, acc, c, 7, dtype="f64")
+    base = _run(sm.Plan(dims, acc, c, "f64", 0), u0, "f64", 7)
+    p = sm.Plan(dims, acc, c, "f64", sm.oc_from_name("ST_TB_BM_RT_PR"), {"tb_steps": 4, "merge": 2})
+    assert p.info["xshift"]
+    got = _run(p, u0, "f64", 7)
+    assert _relerr(got, ref) <= TOL["f64"]
+    assert np.array_equal(got, base)
+
+
 @pytest.mark.parametrize("name,dims,dtype,oc,prm", [
     ("heat3d", (20, 100, 200), "f64", "ST_TB_BM_RT_PR", None),
     ("heat3d", (21, 90, 170), "f64", "ST_TB_CM_RT", {"merge": 4, "by": 4}),
@@ -303,6 +319,9 @@ def test_tb_rt_pipeline_settings(gpu, name, dims, dtype):
     ("random3d:2:5", (22, 70, 140), "f64", "ST_TB_BM_RT_PR", {"tb_steps": 3, "merge": 2}),
     # order-1 Algorithm-1 stencils take the aligned-window ring geometry (xshift)
     ("random3d:1:0", (20, 100, 200), "f64", "ST_TB_BM_RT_PR", None),
+    # T = 4 with xshift: 4 steps in one launch (the remainder-depth guard is in
+    # test_tb_rt_xshift_remainder)
+    ("random3d:1:2", (24, 60, 140), "f64", "ST_TB_BM_RT_PR", {"tb_steps": 4, "merge": 2}),
     ("random3d:1:1", (23, 75, 150), "f64", "ST_TB_CM_RT_PR", {"merge": 2, "by": 8})])
 def test_tb_rt_interior_and_edge_tiles(gpu, name, dims, dtype, oc, prm):
     """k_stream_tb_rt on grids large enough that some tiles lie wholly inside
