@@ -282,6 +282,41 @@ def kernel_key(config: str, lowered: str) -> str:
     return f"{config}:{name}<{','.join(args)}>"
 
 
+def _pcie_probe(hin, hout, x, y):
+    """Host-link context for e2e: one grid up, one grid down, and both at once
+    (two streams), timed with CUDA events -- the bound the pipelined host path
+     works against."""
+    import torch
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    nb = x.numel() * x.element_size()
+
+    def timed(fn):
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        fn()
+        for s in (s1, s2):
+            torch.cuda.current_stream().wait_stream(s)
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) * 1e-3
+
+    def up():
+        with torch.cuda.stream(s1):
+            x.copy_(hin, non_blocking=True)
+
+    def down():
+        with torch.cuda.stream(s2):
+            hout.copy_(y, non_blocking=True)
+
+    for s in (s1, s2):
+        s.wait_stream(torch.cuda.current_stream())
+    t_up, t_down = timed(up), timed(down)
+    t_both = timed(lambda: (up(), down()))
+    return {"h2d": round(nb / t_up / 1e9, 1), "d2h": round(nb / t_down / 1e9, 1),
+            "both_directions_total": round(2 * nb / t_both / 1e9, 1)}
+
+
 def _traffic_from_profiles(key: str):
     """dram read+write bytes per launch from a committed `ncu --set full` capture."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -515,7 +550,9 @@ def run_impl(args):
             e2e_ms = float(t.item())
         nbytes = x.numel() * elem * len(items)
         e2e = {"value": round(pts_all * steps / (e2e_ms * 1e-3) / 1e9, 3), "unit": "GStencil/s",
-               "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes, "ms_per_step": round(e2e_ms, 3)}
+               "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes, "ms_per_step": round(e2e_ms, 3),
+               "host_chunks": [it["plan"].info["host_chunks"] for it in items],
+               "pcie_gbs": _pcie_probe(hin, hout, x, y)}
         del hin, hout
 
     # ---- 5. CPU oracle beside it (rank 0, N = 1)

@@ -111,6 +111,7 @@ typedef struct {
                                  producer/intermediate-stage warps and of the last-stage warps
                                  after setmaxnreg (0, 0 = no split) */
     int32_t xshift;           /* ST_TB_RT kernel uses the aligned-window ring geometry (§6.1) */
+    int32_t host_chunks;      /* z-chunks of the last stencil_run_host (0 = not pipelined) */
 } stencil_plan_info_t;
 
 /* ---------------------------------------------------------------------------

@@ -59,7 +59,8 @@ class PlanInfo(ctypes.Structure):
                 ("params", Params), ("kernel_family", ctypes.c_int32), ("smem_bytes", ctypes.c_int32),
                 ("threads", ctypes.c_int32), ("regs", ctypes.c_int32), ("uses_tma", ctypes.c_int32),
                 ("points", ctypes.c_int64), ("kernel_name", ctypes.c_char * 128),
-                ("reg_split", ctypes.c_int32 * 2), ("xshift", ctypes.c_int32)]
+                ("reg_split", ctypes.c_int32 * 2), ("xshift", ctypes.c_int32),
+                ("host_chunks", ctypes.c_int32)]
 
 
 class Features(ctypes.Structure):
@@ -370,6 +371,7 @@ class Plan:
             "kernel_name": i.kernel_name.decode(),
             "reg_split": (i.reg_split[0], i.reg_split[1]),
             "xshift": bool(i.xshift),
+            "host_chunks": i.host_chunks,
         }
 
     @property

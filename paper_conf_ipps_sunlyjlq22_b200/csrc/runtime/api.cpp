@@ -969,6 +969,7 @@ static int run_host_pipelined(stencil_plan_s* P, const void* hin, void* hout, in
   SM_CUDA(cudaGetLastError());
   SM_CUDA(cudaStreamSynchronize(P->d2h_stream));
   SM_CUDA(cudaStreamSynchronize(P->stream));
+  P->host_chunks = K;
   *done = true;
   return STENCIL_OK;
 }
@@ -1176,6 +1177,7 @@ int stencil_plan_info(stencil_plan_t P, stencil_plan_info_t* info) {
   info->reg_split[0] = P->var.reg_lo;
   info->reg_split[1] = P->var.reg_hi;
   info->xshift = P->var.xshift ? 1 : 0;
+  info->host_chunks = P->host_chunks;
   return STENCIL_OK;
 }
 
@@ -1241,6 +1243,7 @@ int stencil_run_host(stencil_plan_t P, const void* in_host, void* out_host, int 
   {
     bool done = false;
     const char* np = getenv("STENCIL_NO_PIPELINE");   // dev override: unpipelined path
+    P->host_chunks = 0;
     const int rc = (np && atoi(np)) ? STENCIL_OK : run_host_pipelined(P, in_host, out_host, steps, &done);
     if (rc != STENCIL_OK || done) {
       P->ws = saved_ws;

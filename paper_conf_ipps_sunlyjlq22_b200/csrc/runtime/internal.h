@@ -208,6 +208,7 @@ struct stencil_plan_s {
   void* h_ws_dev = nullptr;
   cudaStream_t h2d_stream = nullptr, d2h_stream = nullptr;   // pipelined stencil_run_host
   std::vector<cudaEvent_t> h2d_ev, cmp_ev;
+  int host_chunks = 0;           // chunks of the last stencil_run_host (0 = not pipelined)
 
   // rows of the last OC sweep (stencil_sweep_rows)
   std::vector<stencil_sweep_row_t> sweep_rows;
