@@ -892,8 +892,10 @@ static int run_group(const std::vector<stencil_plan_s*>& Ps, const std::vector<c
 // stencil_run: bitwise equal results. *done = false: the plan does not qualify.
 static int run_host_pipelined(stencil_plan_s* P, const void* hin, void* hout, int steps, bool* done) {
   *done = false;
-  const int nz = (int)P->vdims[0];
-  const int E = std::max(P->pat.zlo, P->pat.zhi);
+  // chunk axis: the slowest view axis, or y for the 2-D tiled/naive views [1][ny][nx]
+  const bool yax = P->vdims[0] == 1;
+  const int nz = (int)(yax ? P->vdims[1] : P->vdims[0]);
+  const int E = yax ? std::max(P->pat.ylo, P->pat.yhi) : std::max(P->pat.zlo, P->pat.zhi);
   if (P->comm || steps < 1 || P->timing || nz < 64) return STENCIL_OK;
   const int T = P->var.family == FAM_TILED || P->var.family == FAM_STREAM_TB ? P->var.tt : 1;
   const int launches = (steps + T - 1) / T;
@@ -904,7 +906,7 @@ static int run_host_pipelined(stencil_plan_s* P, const void* hin, void* hout, in
   if (K < 2) return STENCIL_OK;
   SM_TRY(ensure_loaded(P));
   const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
-  const size_t pb = (size_t)P->vdims[1] * P->vdims[2] * elem;
+  const size_t pb = (yax ? (size_t)P->vdims[2] : (size_t)P->vdims[1] * P->vdims[2]) * elem;   // bytes per plane / row
   char* din = (char*)P->h_in_dev;
   char* dout = (char*)P->h_out_dev;
   char* dws = (char*)P->ws;
@@ -922,6 +924,7 @@ static int run_host_pipelined(stencil_plan_s* P, const void* hin, void* hout, in
   SM_CUDA(cudaStreamWaitEvent(P->h2d_stream, P->cmp_ev[0], 0));
   SM_CUDA(cudaStreamWaitEvent(P->d2h_stream, P->cmp_ev[0], 0));
   const GridArg g = make_grid(P, P->var.vx);
+  const int gc0 = yax ? g.cy0 : g.cz0, gc1 = yax ? g.cy1 : g.cz1;   // compute box along the chunk axis
   std::vector<Variant> vs(launches);
   std::vector<Kernel> ks(launches);
   for (int i = 0; i < launches; ++i) {
@@ -938,21 +941,26 @@ static int run_host_pipelined(stencil_plan_s* P, const void* hin, void* hout, in
     SM_CUDA(cudaStreamWaitEvent(P->stream, P->h2d_ev[k], 0));
     // a4 for these planes: the frame into every buffer the sweep writes
     GridArg gf = g;
-    gf.nz = z1 - z0;
-    gf.uz0 = std::min(std::max(g.uz0 - z0, 0), gf.nz);
-    gf.uz1 = std::min(std::max(g.uz1 - z0, gf.uz0), gf.nz);
+    if (yax) {
+      gf.ny = z1 - z0;
+      gf.uy0 = std::min(std::max(g.uy0 - z0, 0), gf.ny);
+      gf.uy1 = std::min(std::max(g.uy1 - z0, gf.uy0), gf.ny);
+    } else {
+      gf.nz = z1 - z0;
+      gf.uz0 = std::min(std::max(g.uz0 - z0, 0), gf.nz);
+      gf.uz1 = std::min(std::max(g.uz1 - z0, gf.uz0), gf.nz);
+    }
     SM_TRY(launch_frame_copy(din + z0 * pb, dout + z0 * pb, elem, gf, P->stream));
     if (launches >= 2) SM_TRY(launch_frame_copy(din + z0 * pb, dws + z0 * pb, elem, gf, P->stream));
     const void* src = din;
     for (int i = 0; i < launches; ++i) {
       const int sk = (i + 1) * T * E;
       char* dst = ((launches - 1 - i) % 2 == 0) ? dout : dws;
-      const int lo = std::max(g.cz0, k == 0 ? 0 : z0 - sk);
-      const int hi = std::min(g.cz1, k == K - 1 ? nz : z1 - sk);
+      const int lo = std::max(gc0, k == 0 ? 0 : z0 - sk);
+      const int hi = std::min(gc1, k == K - 1 ? nz : z1 - sk);
       if (hi > lo) {
         GridArg gl = g;
-        gl.cz0 = lo;
-        gl.cz1 = hi;
+        if (yax) { gl.cy0 = lo; gl.cy1 = hi; } else { gl.cz0 = lo; gl.cz1 = hi; }
         SM_TRY(launch_sweep(P, vs[i], ks[i], src, dst, gl));
       }
       src = dst;

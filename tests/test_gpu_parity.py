@@ -187,7 +187,10 @@ def test_run_host_end_to_end(gpu):
     ("random3d:1:0", (140, 40, 80), "f64", "ST_TB_CM_RT", {"merge": 2}, 6),
     ("star25", (200, 30, 72), "f32", "ST_RT_PR", None, 2),
     ("box125", (128, 26, 40), "f64", "TB_BM", {"tb_steps": 2}, 3),
-    ("random2d:3:8", (700, 90), "f64", "ST_BM_RT_PR", None, 4)])
+    ("random2d:3:8", (700, 90), "f64", "ST_BM_RT_PR", None, 4),
+    # 2-D tiled / naive views [1][ny][nx] chunk along y
+    ("random2d:1:0", (600, 130), "f64", "TB_BM", None, 5),
+    ("random2d:2:4", (300, 100), "f64", "base", None, 3)])
 def test_run_host_pipelined(gpu, name, dims, dtype, oc, prm, steps):
     """stencil_run_host pipelines H2D / sweep / D2H over z-chunks with a
     time-skewed wavefront (api.cpp run_host_pipelined): bitwise equal to the
