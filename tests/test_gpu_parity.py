@@ -202,6 +202,7 @@ def test_run_host_pipelined(gpu, name, dims, dtype, oc, prm, steps):
     p = sm.Plan(dims, acc, c, dtype, sm.oc_from_name(oc), prm)
     out = np.empty_like(u0)
     p.run_host(u0, out, steps)
+    assert p.info["host_chunks"] >= 2          # the pipelined path ran
     dev = _run(p, u0, dtype, steps)
     assert np.array_equal(out, dev)
     os.environ["STENCIL_NO_PIPELINE"] = "1"
