@@ -2,6 +2,9 @@
 
 Algorithm 1 is random, so it is pinned by invariants G1-G4.
 """
+import itertools
+import math
+
 import numpy as np
 import pytest
 
@@ -78,3 +81,71 @@ def test_algorithm1_full_box_and_determinism(ndim):
     a1, _ = si.random_stencil(ndim, 3, 123)
     a2, _ = si.random_stencil(ndim, 3, 123)
     assert np.array_equal(a1, a2)
+
+
+def _moore_ring(points, ndim, k):
+    """Independent Moore-neighbourhood expansion (itertools), restricted to ring k."""
+    out = set()
+    for q in points:
+        for d in itertools.product((-1, 0, 1), repeat=ndim):
+            if any(d):
+                c = tuple(a + b for a, b in zip(q, d))
+                if max(abs(v) for v in c) == k:
+                    out.add(c)
+    return out
+
+
+def _trunc_binom(n, p):
+    """Mean and variance of Binomial(n, p) conditioned on >= 1 success (the
+    redraw of reading C-7)."""
+    z = 1.0 - (1.0 - p) ** n
+    m1 = n * p / z
+    m2 = (n * p * (1.0 - p) + (n * p) ** 2) / z
+    return m1, m2 - m1 * m1
+
+
+@pytest.mark.parametrize("ndim,samples", [(2, 3000), (3, 1500)])
+def test_algorithm1_order1_distribution(ndim, samples):
+    """G5 (Alg. 1 lines 4-6; reading C-7): at order 1 every one of
+    the 3^d - 1 Moore neighbours of the centre is a candidate and is kept with
+    probability p / (1 - (1-p)^M); the ring-1 count is a truncated binomial.
+    A star-only neighbourhood or a biased draw fails here."""
+    M = 3 ** ndim - 1
+    p = 0.5
+    pk = p / (1.0 - (1.0 - p) ** M)
+    freq = {}
+    counts = []
+    for s in range(samples):
+        _, np_list = si.random_stencil(ndim, 1, 10_000 + s)
+        counts.append(len(np_list[0]))
+        for q in np_list[0]:
+            freq[q] = freq.get(q, 0) + 1
+    assert set(freq) == _moore_ring([(0,) * ndim], ndim, 1)
+    sd = math.sqrt(pk * (1 - pk) / samples)
+    for q, f in freq.items():
+        assert abs(f / samples - pk) < 5 * sd, (q, f / samples, pk)
+    m, v = _trunc_binom(M, p)
+    assert abs(np.mean(counts) - m) < 5 * math.sqrt(v / samples)
+
+
+@pytest.mark.parametrize("ndim,order,samples", [(2, 2, 1500), (3, 2, 600), (2, 3, 800), (3, 3, 300)])
+def test_algorithm1_higher_order_conditional_counts(ndim, order, samples):
+    """G6 (Alg. 1 lines 8-14): given the order-(k-1) selection S,
+    the ring-k candidates are exactly the Moore neighbours of S lying on ring k
+    (rings k-1 and k-2 deleted), each kept with probability p under the redraw
+    of reading C-7. Summed over samples, (count - E[count | S]) is centred with
+    the truncated-binomial variance: candidates drawn from only part of S (e.g.
+    the previous ring's axis points) or a different keep probability shift the
+    mean by many sigmas. Ring deletion itself is pinned by G2/G3 above."""
+    p = 0.5
+    dev, var = 0.0, 0.0
+    for s in range(samples):
+        _, np_list = si.random_stencil(ndim, order, 20_000 + s)
+        prev = np_list[order - 2]
+        cand = _moore_ring(prev, ndim, order)
+        got = [q for q in np_list[order - 1] if si.ring_index(q) == order]
+        assert set(got) <= cand
+        m, v = _trunc_binom(len(cand), p)
+        dev += len(got) - m
+        var += v
+    assert abs(dev) < 5 * math.sqrt(var)
