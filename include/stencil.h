@@ -174,7 +174,8 @@ int stencil_run(stencil_plan_t plan, const void *in_dev, void *out_dev, int step
  * memory for full PCIe speed). The call copies in_host to device buffers it
  * owns, runs `steps` steps with the plan's OC, copies the result back and
  * returns when out_host holds it (the plan's stream is synchronised). Single-GPU
- * plans whose slowest view axis has >= 64 planes are pipelined over z-chunks:
+ * plans whose slowest view axis has >= 64 planes and whose grid holds >= 32 MiB
+ * are pipelined over z-chunks:
  * the upload of chunk k+1, a time-skewed sweep of chunk k and the download of
  * chunk k-1 overlap on two internal copy streams; the result is bitwise that of
  * stencil_run. Errors as stencil_run. */

@@ -906,9 +906,15 @@ static int run_host_pipelined(stencil_plan_s* P, const void* hin, void* hout, in
   // twice the skew (the wavefront must stay well inside a chunk)
   const int K = (int)std::min<long long>(16, nz / std::max<long long>(32, 2 * skew + 1));
   if (K < 2) return STENCIL_OK;
-  SM_TRY(ensure_loaded(P));
   const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
   const size_t pb = (yax ? (size_t)P->vdims[2] : (size_t)P->vdims[1] * P->vdims[2]) * elem;   // bytes per plane / row
+  // small grids: ~3 copies/launches of ~10 us per chunk outweigh the overlap
+  // (C1 256^2 fp64: 0.10 ms unpipelined, 0.48 ms in 8 chunks); the pipeline
+  // pays from tens of MB (copy time ~ bytes / 50 GB/s). Dev override for tests.
+  const char* mb = getenv("STENCIL_PIPELINE_MIN_BYTES");
+  const size_t min_bytes = mb ? (size_t)atoll(mb) : ((size_t)32 << 20);
+  if (pb * (size_t)nz < min_bytes) return STENCIL_OK;
+  SM_TRY(ensure_loaded(P));
   char* din = (char*)P->h_in_dev;
   char* dout = (char*)P->h_out_dev;
   char* dws = (char*)P->ws;

@@ -201,7 +201,11 @@ def test_run_host_pipelined(gpu, name, dims, dtype, oc, prm, steps):
     u0 = np.ascontiguousarray(si.make_field(dims, 17, dtype))
     p = sm.Plan(dims, acc, c, dtype, sm.oc_from_name(oc), prm)
     out = np.empty_like(u0)
-    p.run_host(u0, out, steps)
+    os.environ["STENCIL_PIPELINE_MIN_BYTES"] = "0"     # these grids are below the size threshold
+    try:
+        p.run_host(u0, out, steps)
+    finally:
+        del os.environ["STENCIL_PIPELINE_MIN_BYTES"]
     assert p.info["host_chunks"] >= 2          # the pipelined path ran
     dev = _run(p, u0, dtype, steps)
     assert np.array_equal(out, dev)
