@@ -180,6 +180,21 @@ def test_run_host_end_to_end(gpu):
     assert _relerr(out, ref) <= 1e-5
 
 
+def test_run_host_small_grid_not_pipelined(gpu):
+    """C1-sized grids (256^2 fp64, 0.5 MB) stay on the unpipelined host path:
+    per-chunk copy/launch latency would exceed the overlap (api.cpp
+    run_host_pipelined size threshold)."""
+    acc, c = si.heat2d()
+    dims = (256, 256)
+    u0 = np.ascontiguousarray(si.make_field(dims, 3, "f64"))
+    p = sm.Plan(dims, acc, c, "f64", sm.OC_ST | sm.OC_RT)
+    out = np.empty_like(u0)
+    p.run_host(u0, out, 10)
+    assert p.info["host_chunks"] == 0
+    ref = oracle.sweep(u0, acc, c, 10, dtype="f64")
+    assert _relerr(out, ref) <= 1e-12
+
+
 @pytest.mark.parametrize("name,dims,dtype,oc,prm,steps", [
     ("heat3d", (160, 40, 72), "f64", "ST_TB_BM_RT_PR", None, 5),      # TB with a remainder launch
     ("heat3d", (130, 33, 64), "f64", "base", None, 4),
