@@ -1,10 +1,14 @@
 #!/usr/bin/env python
 """bench.py -- GStencil/s and % of HBM roofline per OC on B200 (BASELINE.json metric).
 
-Default workload (BASELINE.json configs[1], "C2"): the 3-D 7-point heat stencil
-(order 1) on a 512^3 fp64 grid, 10 time steps, under every OC of Table I.
+Default workload ("C5", BASELINE.json configs[4]): the configuration the metric
+is quoted on ("... per OC at 1/2/4/8 B200") and the largest per-GPU one -- four
+random Algorithm-1 3-D stencils, one per order r = 1..4, 1024^3 fp64 per GPU,
+4 time steps each, every OC of Table I swept per stencil, z-slabs with the halo
+exchange at N > 1 (weak scaling). `--config C1..C4, N2` select the others.
 
-What one run does (one process per GPU; torchrun for N > 1):
+What one run does (one process per GPU: torchrun, or `--gpus N` spawns the N
+ranks itself):
   1. label pass: stencil_oc_sweep over the 30 OCs with the
      library's seeded settings; its per-OC times give "per_oc" (GStencil/s and
      HBM fraction of every OC) and the label (best OC + its setting);
@@ -16,7 +20,9 @@ What one run does (one process per GPU; torchrun for N > 1):
   3. roofline of the dominant kernel (the labelled OC's sweep kernel): bytes a
      launch must move (read + write the grid once: 16 B / point in fp64, for
      every fused step count) / its average launch duration, from CUDA events
-     around each launch over the timed region;
+     around each launch over the timed region -- or, for FMA-bound stencils,
+     flops / time against the FMA peak measured in the same run
+     (stencil_fma_probe, `fma_peak`);
   4. e2e: the same metric through stencil_run_host (pinned host buffers in,
      H2D + 10 steps + D2H inside the timed region);
   5. cpu_baseline: the oracle (oracle/, plain C loops, OpenMP) on a bounded
@@ -169,13 +175,24 @@ def cpu_oracle_sample(name: str, budget_s: float = 12.0, acc=None, c=None):
     r = (acc.shape[0] - 1) // 2
     threads = oracle.max_threads()
     if len(dims) == 2 and dims[0] * dims[1] <= 1 << 20:
+        # small 2-D grid (C1): the whole workload, "CPU oracle in seconds" with 1
+        # thread and with every thread (best of 5 each)
         u = si.make_field(dims, C["seed"], dtype)
-        t0 = time.perf_counter()
-        oracle.sweep(u, acc, c, steps, dtype=dtype)
-        dt = time.perf_counter() - t0
+        secs = {}
+        for nt in (1, threads):
+            best = math.inf
+            for _ in range(5):
+                t0 = time.perf_counter()
+                oracle.sweep(u, acc, c, steps, dtype=dtype, nthreads=nt)
+                best = min(best, time.perf_counter() - t0)
+            secs[nt] = best
+        dt = secs[threads]
         pts = (dims[0] - 2 * r) * (dims[1] - 2 * r) * steps
         return {"value": pts / dt / 1e9, "unit": "GStencil/s", "cores": threads, "kind": "oracle",
-                "sample": f"full {name} grid {dims}, {steps} steps, {dt:.2f} s", "seconds": dt, "points": pts}
+                "sample": (f"full {name} grid {dims}, {steps} steps: {secs[1]:.6f} s on 1 thread, "
+                           f"{dt:.6f} s on {threads} threads (best of 5)"),
+                "seconds": dt, "points": pts, "seconds_1_thread": round(secs[1], 6),
+                "seconds_all_threads": round(dt, 6), "cpu_model": _cpu_model()}
     # probe with a thin slab (rows in 2-D, planes in 3-D), then size the sample to ~budget_s
     row = tuple(dims[1:])
     nz = 2 * r + 8
@@ -203,6 +220,16 @@ def cpu_oracle_sample(name: str, budget_s: float = 12.0, acc=None, c=None):
                        f"{dt:.2f} s; rate per interior update"), "seconds": dt, "points": pts}
 
 
+def _cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 def _cpu_workload(name: str, budget_s: float):
     """Oracle rate over every stencil of the workload: total sampled updates /
     total seconds (the same aggregation as the GPU value)."""
@@ -224,8 +251,12 @@ def _cpu_workload(name: str, budget_s: float):
     v = tot_pts / tot_s / 1e9
     sample = "; ".join(f"{it['stencil']}: {x['sample']}" for it, x in zip(items, samples)) if len(items) > 1 \
         else samples[0]["sample"]
-    return {"value": v, "unit": "GStencil/s", "cores": samples[0]["cores"], "kind": "oracle", "sample": sample,
-            "seconds": sec, "points": pts}
+    out = {"value": v, "unit": "GStencil/s", "cores": samples[0]["cores"], "kind": "oracle", "sample": sample,
+           "seconds": sec, "points": pts, "cpu_model": _cpu_model()}
+    for k in ("seconds_1_thread", "seconds_all_threads"):
+        if k in samples[0]:
+            out[k] = samples[0][k]
+    return out
 
 
 def _workload_points(name: str) -> int:
@@ -262,7 +293,8 @@ def run_reference(args):
         "config": {"workload": WORKLOADS.get(name, name), "grid": list(C["dims"]), "time_steps": C["steps"],
                    "stencils": [it["stencil"] for it in _items(name)],
                    "note": "oracle timed on a bounded slab sample; ms_per_step extrapolated to the full grid"},
-        "cpu_baseline": {k: cb[k] for k in ("kind", "cores", "sample")} | {"value": v, "unit": "GStencil/s"},
+        "cpu_baseline": {k: cb[k] for k in ("kind", "cores", "sample", "cpu_model", "seconds_1_thread",
+                                            "seconds_all_threads") if k in cb} | {"value": v, "unit": "GStencil/s"},
         "e2e": {"value": v, "unit": "GStencil/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -329,7 +361,46 @@ def _traffic_from_profiles(key: str):
         return None
 
 
-def _roofline(name, sm, pinfo, oc, pts, steps, kern_ms, kern_n, total_ms, nsteps_timed, elem, dtype, peak, peak_kind):
+def measure_fma_peak(sm, dtype: str, local: int, seconds: float = 2.0) -> dict:
+    """Measured FMA throughput of this GPU in `dtype` (stencil_fma_probe, a
+    hand-written kernel of independent FMA chains on every SM): back-to-back
+    launches of ~20 ms for `seconds`, SM clock sampled meanwhile. `sustained`
+    (median of the second half, under the power cap) is the denominator of the
+    "alu" roofline -- the FMA-bound stencil kernels are timed inside a long
+    step; `burst` is the best launch."""
+    import torch
+    tdt = torch.float64 if dtype == "f64" else torch.float32
+    sink = torch.zeros(1, dtype=tdt, device=f"cuda:{local}")
+    stream = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+
+    def once(iters):
+        e0.record(stream)
+        fl = sm.fma_probe(sink, iters, stream=stream)
+        e1.record(stream)
+        e1.synchronize()
+        ms = e0.elapsed_time(e1)
+        return fl / (ms * 1e-3) / 1e12, ms
+
+    iters = 256
+    once(iters)
+    _, ms = once(iters)
+    iters = max(1, int(iters * 20.0 / max(ms, 1e-3)))
+    vals = []
+    with ClockSampler(local) as clk:
+        t_end = time.time() + seconds
+        while time.time() < t_end or len(vals) < 6:
+            vals.append(once(iters)[0])
+    half = vals[len(vals) // 2:]
+    c = clk.result()
+    return {"sustained": round(statistics.median(half), 2), "burst": round(max(vals), 2), "unit": "TFLOP/s",
+            "dtype": dtype, "launches": len(vals), "sm_mhz": c["sm_mhz"], "reasons": c["reasons"],
+            "how": "stencil_fma_probe: 148 SMs x 8 CTAs x 256 threads, 8 independent FMA chains per thread, "
+                   "~20 ms launches back to back; 2 flops per FMA"}
+
+
+def _roofline(name, sm, pinfo, oc, pts, steps, kern_ms, kern_n, total_ms, nsteps_timed, elem, dtype, peak, peak_kind,
+              fma_peak=None):
     """Roofline of one stencil's sweep kernel: algorithmic bytes
     per launch (read + write every interior point once) / average launch time,
     and the FMA ceiling; the binding one is reported."""
@@ -339,8 +410,15 @@ def _roofline(name, sm, pinfo, oc, pts, steps, kern_ms, kern_n, total_ms, nsteps
     flops_per_step = pts * 2 * pinfo["nnz"]    # one FMA per neighbour per point and step
     avg_launch_ms = kern_ms / max(groups, 1)
     achieved = bytes_per_launch / (avg_launch_ms * 1e-3) / 1e9
-    # FP64 148 SM x 64 FMA/clk x 2 x 1.965 GHz = 37.2 TFLOP/s; FP32 x2
-    fp_peak = 148 * 64 * 2 * 1.965e9 / 1e12 * (1 if dtype == "f64" else 2)
+    # measured FMA peak (stencil_fma_probe, sustained); fallback: DESIGN.md §6's
+    # derived 148 SM x 64 FMA/clk x 2 x 1.965 GHz = 37.2 TFLOP/s (FP32 x2)
+    if fma_peak:
+        fp_peak = fma_peak["sustained"]
+        fp_kind = (f"measured (stencil_fma_probe, sustained, SM clock median {fma_peak['sm_mhz']} MHz; "
+                   f"burst {fma_peak['burst']})")
+    else:
+        fp_peak = 148 * 64 * 2 * 1.965e9 / 1e12 * (1 if dtype == "f64" else 2)
+        fp_kind = "derived (DESIGN.md §6)"
     achieved_fp = flops_per_step * nsteps_timed * steps / (kern_ms * 1e-3) / 1e12
     key = kernel_key(name, pinfo["kernel_name"])
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
@@ -351,12 +429,12 @@ def _roofline(name, sm, pinfo, oc, pts, steps, kern_ms, kern_n, total_ms, nsteps
             "bytes_per_launch": bytes_per_launch, "time_steps_per_launch": T,
             "frac_of_spec_8tbs": round(achieved / HBM_SPEC_GBS, 4),
             "fp": {"achieved": round(achieved_fp, 2), "peak": round(fp_peak, 1), "unit": "TFLOP/s",
-                   "frac": round(achieved_fp / fp_peak, 4), "peak_kind": "derived (DESIGN.md §6)"}}
+                   "frac": round(achieved_fp / fp_peak, 4), "peak_kind": fp_kind}}
     # FMA-bound stencils (C4, high-order random): the FP ceiling binds before HBM
     if flops_per_step / (fp_peak * 1e12) > bytes_per_launch / T / (peak * 1e9):
         roof.update({"bound": "alu", "achieved": round(achieved_fp, 2), "peak": round(fp_peak, 1),
                      "unit": "TFLOP/s", "frac": round(achieved_fp / fp_peak, 4),
-                     "peak_kind": "derived (DESIGN.md §6)",
+                     "peak_kind": fp_kind,
                      "hbm": {"achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                              "frac": round(achieved / peak, 4)}})
         roof.pop("fp")
@@ -369,6 +447,8 @@ def run_impl(args):
     import paper_conf_ipps_sunlyjlq22_b200 as sm
 
     rank, world, local = _env_rank()
+    assert world == args.gpus, f"WORLD_SIZE={world} != --gpus {args.gpus}"
+    assert torch.cuda.device_count() > local, f"rank {rank}: no GPU {local}"
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
@@ -441,11 +521,15 @@ def run_impl(args):
             if oc not in ocs:
                 continue
             gs = sm.gstencil_per_s(it["points"], steps, t) if math.isfinite(t) else None
+            # a launch reads and writes the grid once (16 B / point in fp64) whatever
+            # number of time steps it fuses: TB OCs move 2*elem/T bytes per update
+            T_oc = (p or {}).get("tb_steps", 1) if oc & sm.OC_TB else 1
             per_oc[sm.oc_name(oc)] = {
                 "ms": round(t, 4) if math.isfinite(t) else None,
                 "gstencil_s": round(gs, 2) if gs else None,
-                "hbm_frac_of_measured": round(gs * 2 * elem / peak, 4) if gs else None,
-                "hbm_frac_of_spec": round(gs * 2 * elem / HBM_SPEC_GBS, 4) if gs else None,
+                "time_steps_per_launch": T_oc,
+                "hbm_frac_of_measured": round(gs * 2 * elem / T_oc / peak, 4) if gs else None,
+                "hbm_frac_of_spec": round(gs * 2 * elem / T_oc / HBM_SPEC_GBS, 4) if gs else None,
                 "infeasible": not math.isfinite(t),
             }
             if math.isfinite(t) and t < best_t:
@@ -482,6 +566,9 @@ def run_impl(args):
         t = torch.tensor([pts_rank], dtype=torch.float64, device=dev)
         dist.all_reduce(t)
         pts_all = int(t.item())
+
+    # measured FMA peak (the "alu" roofline's denominator), before the timed region
+    fma_peak = measure_fma_peak(sm, dtype, local)
 
     def step():
         for it in items:
@@ -522,15 +609,23 @@ def run_impl(args):
     # ---- 3. roofline per stencil; the dominant kernel (largest share of the step) is reported
     for it in items:
         it["roofline"] = _roofline(name, sm, it["pinfo"], it["best_oc"], it["points"], steps, it["kern_ms"],
-                                   it["kern_n"], total_ms, args.steps, elem, dtype, peak, peak_kind)
+                                   it["kern_n"], total_ms, args.steps, elem, dtype, peak, peak_kind, fma_peak)
     dom = max(items, key=lambda it: it["kern_ms"])
     roofline = dict(dom["roofline"])
     if len(items) > 1:
         roofline["stencil"] = dom["stencil"]
 
+    launch_bytes = sum(it["points"] * 2 * elem * math.ceil(steps / it["roofline"]["time_steps_per_launch"])
+                       for it in items)
+    hbm_gbs = launch_bytes / (ms_per_step * 1e-3) / 1e9
+
     # ---- 4. e2e through the public API with host buffers
     e2e = None
-    if not args.no_e2e:
+    if slab and args.transport == "p2p" and not args.no_e2e:
+        # P2P slab plans run only on their registered buffers: the host path
+        # (which stages into its own device buffers) does not apply
+        e2e = {"value": None, "unsupported": "stencil_run_host does not run P2P-registered slab plans"}
+    elif not args.no_e2e:
         hin = torch.empty(tuple(x.shape), dtype=tdt, pin_memory=True)
         hin.copy_(x.cpu())
         hout = torch.empty_like(hin).pin_memory()
@@ -559,7 +654,8 @@ def run_impl(args):
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         cb = _cpu_workload(name, args.cpu_budget)
-        cpu = {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample")}
+        cpu = {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample", "cpu_model", "seconds_1_thread",
+                                  "seconds_all_threads") if k in cb}
 
     if rank == 0:
         first = items[0]
@@ -582,8 +678,11 @@ def run_impl(args):
                                        if slab else "single GPU"),
                        "l2": "inputs (grid bytes) larger than the 126 MB L2; no flush needed"},
             "roofline": roofline,
-            "hbm_frac_of_measured_per_gpu": round(value / world * 2 * elem / peak, 4),
-            "hbm_frac_of_spec_per_gpu": round(value / world * 2 * elem / HBM_SPEC_GBS, 4),
+            # algorithmic bytes per step (every launch reads + writes its grid once;
+            # TB launches fuse T steps) / step time, per GPU
+            "hbm_frac_of_measured_per_gpu": round(hbm_gbs / peak, 4),
+            "hbm_frac_of_spec_per_gpu": round(hbm_gbs / HBM_SPEC_GBS, 4),
+            "fma_peak": fma_peak,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches,
@@ -614,7 +713,8 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5", "N2"])
+    ap.add_argument("--config", default="C5", choices=["C1", "C2", "C3", "C4", "C5", "N2"],
+                    help="workload (default C5: the configuration BASELINE.json's metric is quoted on)")
     ap.add_argument("--settings", type=int, default=None,
                     help="settings per OC in the label pass (default 3; C5: 1, N2: 2)")
     ap.add_argument("--seed", type=int, default=0)
@@ -634,7 +734,33 @@ def main():
         args.settings = {"C5": 1, "N2": 2}.get(args.config, 3)
     if args.impl == "reference":
         return run_reference(args)
+    world_env = os.environ.get("WORLD_SIZE")
+    if world_env is None and args.gpus > 1:
+        return spawn_ranks(args)
+    if int(world_env or 1) != args.gpus:
+        ap.error(f"--gpus {args.gpus} but WORLD_SIZE={world_env}: launch one rank per GPU")
     return run_impl(args)
+
+
+def _rank_entry(local: int, args, port: int):
+    os.environ.update(RANK=str(local), LOCAL_RANK=str(local), WORLD_SIZE=str(args.gpus),
+                      MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    rc = run_impl(args)
+    if rc:
+        raise SystemExit(rc)
+
+
+def spawn_ranks(args) -> int:
+    """`--gpus N` without torchrun: spawn one process per GPU (NCCL over
+    NVLink), each with RANK / LOCAL_RANK / WORLD_SIZE set as torchrun would;
+    rank 0 prints the line. Fails loudly rather than timing fewer GPUs."""
+    import torch
+    import torch.multiprocessing as mp
+    have = torch.cuda.device_count()
+    if have < args.gpus:
+        raise SystemExit(f"bench.py --gpus {args.gpus}: only {have} GPU(s) visible")
+    mp.spawn(_rank_entry, args=(args, _free_port()), nprocs=args.gpus, join=True)
+    return 0
 
 
 if __name__ == "__main__":

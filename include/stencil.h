@@ -284,6 +284,19 @@ int stencil_oc_analysis(int n_stencils, int n_oc, const double *times, int n_cla
  * Synthetic inputs (the counter-based generator of DESIGN.md, reading C-3)
  * ------------------------------------------------------------------------- */
 
+/* FMA-throughput probe (measurement only): enqueue on
+ * `cuda_stream` one launch of blocks_per_sm (1..8) x SM-count CTAs of 256
+ * threads, each thread running 8 independent fused-multiply-add chains for
+ * iters x 8 steps in `dtype`; *flops receives the launch's floating-point
+ * operations (2 per FMA). The caller times the launch (CUDA events on the same
+ * stream) to get the measured FMA peak that the "alu" roofline of FMA-bound
+ * stencils divides by -- the paper lists each GPU's FP64 peak.
+ * `sink` is a device buffer of at least one element of `dtype` (written only in
+ * a case that never happens; it keeps the chains live). E_INVAL on bad
+ * arguments. */
+int stencil_fma_probe(stencil_dtype_t dtype, int64_t iters, int blocks_per_sm, void *sink, void *cuda_stream,
+                      double *flops);
+
 /* Fill a device box of shape box_dims (ndim values, slowest first) whose
  * element i holds value(h(seed, g)), g = the row-major linear index of
  * (origin + i) in a grid of shape global_dims. kind 0 = uniform in [1,2),

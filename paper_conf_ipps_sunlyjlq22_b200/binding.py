@@ -118,6 +118,8 @@ _SIGS = {
                                           ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64),
                                           ctypes.POINTER(ctypes.c_int64), ctypes.c_uint64, ctypes.c_int,
                                           ctypes.c_void_p]),
+    "stencil_fma_probe": (ctypes.c_int, [ctypes.c_int, ctypes.c_int64, ctypes.c_int, ctypes.c_void_p,
+                                         ctypes.c_void_p, ctypes.POINTER(ctypes.c_double)]),
     "stencil_nccl_unique_id": (ctypes.c_int, [ctypes.c_void_p]),
     "stencil_plan_set_comm": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int, ctypes.c_int]),
     "stencil_slab_range": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int, ctypes.c_int,
@@ -311,6 +313,19 @@ def fill_field(t, seed: int, kind: int = 0, origin: Optional[Sequence[int]] = No
     dt = F64 if t.dtype == torch.float64 else F32
     _check(lib().stencil_fill_field(ctypes.c_void_p(t.data_ptr()), dt, nd, box, org, gd, seed, kind,
                                     ctypes.c_void_p(_stream_ptr(stream))))
+
+
+def fma_probe(sink, iters: int, blocks_per_sm: int = 8, stream=None) -> float:
+    """Enqueue one FMA-throughput probe launch (stencil_fma_probe) in the dtype
+    of the device tensor `sink`; returns the launch's flops (time it with CUDA
+    events on the same stream)."""
+    import torch
+    assert sink.is_cuda and sink.numel() >= 1
+    fl = ctypes.c_double()
+    dt = F64 if sink.dtype == torch.float64 else F32
+    _check(lib().stencil_fma_probe(dt, int(iters), int(blocks_per_sm), ctypes.c_void_p(sink.data_ptr()),
+                                   ctypes.c_void_p(_stream_ptr(stream)), ctypes.byref(fl)))
+    return float(fl.value)
 
 
 # ------------------------------------------------------------------------ plan

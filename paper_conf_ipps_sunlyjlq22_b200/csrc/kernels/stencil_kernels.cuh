@@ -126,6 +126,11 @@ __device__ __forceinline__ void cp_async_zfill(void* dst, const void* src, bool 
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" :: "n"(N) : "memory"); }
+// arrive on `bar` once every cp.async this thread issued so far has landed
+// (the barrier's expected count includes this arrival: .noinc)
+__device__ __forceinline__ void cp_async_mbar_arrive(unsigned long long* bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" :: "r"(smem_u32(bar)) : "memory");
+}
 
 // ---------------------------------------------------------------------------
 // vector access: VX consecutive elements, 128-bit (or 64-bit) accesses
@@ -249,6 +254,24 @@ struct GlobalPlane {                  // global memory through the read-only pat
     for (int e = 0; e < VX; ++e) w[e] = __ldg(q + e);
   }
 };
+
+// Stage the LX x LY box of plane z at (X0, Y0) into shared memory with
+// element-wise cp.async, zero fill outside the array (what the TMA box does):
+// the staging path of the streaming TB kernels when the rows are not 16-byte
+// multiples (no tensor map can describe them) or the box exceeds 256. NT
+// threads, this one is t.
+template <class T, int LX, int LY, int NT>
+__device__ __forceinline__ void stage_plane_cp_async(T* dst, const T* in, const Grid& g, int X0, int Y0, int z,
+                                                     int t) {
+  const bool zok = z >= 0 && z < g.nz;
+  const T* plane = in + (i64)(zok ? z : 0) * g.sz;
+  for (int i = t; i < LX * LY; i += NT) {
+    const int lx = i % LX, ly = i / LX;
+    const int gx = X0 + lx, gy = Y0 + ly;
+    const bool ok = zok && gx >= 0 && gx < g.nx && gy >= 0 && gy < g.ny;
+    cp_async_zfill<sizeof(T)>(dst + i, ok ? plane + (i64)gy * g.sy + gx : in, ok);
+  }
+}
 
 // ---------------------------------------------------------------------------
 // Compute on a thread tile of M rows x VX columns, driven by the op table of
@@ -858,9 +881,13 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
 
   auto issue = [&](int it) {
     const int slot = it % C::NIN;
-    if (tid == 0) {
-      mbar_expect_tx(&bar[slot], C::LX * C::LY * (unsigned)sizeof(T));
-      tma_load_3d(ring0 + slot * C::PLANE, &tmap, &bar[slot], X0, Y0, pin0 + it);
+    if constexpr (S::TMA) {
+      if (tid == 0) {
+        mbar_expect_tx(&bar[slot], C::LX * C::LY * (unsigned)sizeof(T));
+        tma_load_3d(ring0 + slot * C::PLANE, &tmap, &bar[slot], X0, Y0, pin0 + it);
+      }
+    } else {   // rows not TMA-aligned (or box > 256): element-wise cp.async, zero fill outside
+      stage_plane_cp_async<T, C::LX, C::LY, C::THREADS>(ring0 + slot * C::PLANE, in, g, X0, Y0, pin0 + it, tid);
     }
   };
   // plane pointer of stage k (0 = input) holding plane q
@@ -869,15 +896,17 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
     return k == 0 ? ring0 + (idx % C::NIN) * C::PLANE : mid + ((k - 1) * NZ + idx % NZ) * C::PLANE;
   };
 
-  if (tid == 0) {
+  if (S::TMA && tid == 0) {
     tma_prefetch_desc(&tmap);
     for (int s = 0; s < C::NIN; ++s) mbar_init(&bar[s], 1);
     fence_mbar_init();
   }
   __syncthreads();
 #pragma unroll 1
-  for (int it = 0; it < NS - 1; ++it)
+  for (int it = 0; it < NS - 1; ++it) {
     if (it < nit) issue(it);
+    if constexpr (!S::TMA) cp_async_commit();
+  }
 
   // Intermediate fused step s (1..TT-1) of iteration it: plane q = p - s*ZHI
   // on region R_s (tile expanded by (TT-s)*extent), computed in VX x MI
@@ -940,7 +969,13 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
   // one pipeline iteration up to (excluding) the last stage
   auto front = [&](int it) {
     if (it + NS - 1 < nit) issue(it + NS - 1);
-    mbar_wait(&bar[it % C::NIN], (unsigned)((it / C::NIN) & 1));
+    if constexpr (S::TMA) {
+      mbar_wait(&bar[it % C::NIN], (unsigned)((it / C::NIN) & 1));
+    } else {
+      cp_async_commit();
+      cp_async_wait<NS - 1>();
+      __syncthreads();
+    }
     static_for<1, TT>([&](auto sc) {
       mid_stage(it, sc);
       __syncthreads();
@@ -1137,9 +1172,9 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
   // stage planes start defined (their unwritten corners only feed discarded outputs)
   for (int i = tid; i < C::ELEMS; i += C::THREADS) sbase[i] = T(0);
   if (tid == 0) {
-    tma_prefetch_desc(&tmap);
+    if constexpr (S::TMA) tma_prefetch_desc(&tmap);
     for (int q = 0; q < NR; ++q) {
-      mbar_init(&full_in[q], 1);
+      mbar_init(&full_in[q], S::TMA ? 1 : 32);   // cp.async: one arrival per producer lane
       mbar_init(&empty_in[q], 32 * TbRtStage<S, BX, BY, VX, M, TT, MI, 1>::W);
     }
     static_for<1, TT>([&](auto sc) {
@@ -1161,13 +1196,23 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
 
   // ------------------------------------------------------------ producer
   if (warp == 0) {
-    if (tid == 0) {
+    if constexpr (S::TMA) {
+      if (tid == 0) {
+#pragma unroll 1
+        for (int j = 0; j < nin; ++j) {
+          const int slot = j % NR;
+          if (j >= NR) mbar_wait_sleep(&empty_in[slot], (unsigned)((j / NR - 1) & 1));
+          mbar_expect_tx(&full_in[slot], C::LX * C::LY * (unsigned)sizeof(T));
+          tma_load_3d(ring0 + slot * C::PLANE, &tmap, &full_in[slot], X0, Y0, pin0 + j);
+        }
+      }
+    } else {   // rows not TMA-aligned: the whole warp stages planes with cp.async
 #pragma unroll 1
       for (int j = 0; j < nin; ++j) {
         const int slot = j % NR;
         if (j >= NR) mbar_wait_sleep(&empty_in[slot], (unsigned)((j / NR - 1) & 1));
-        mbar_expect_tx(&full_in[slot], C::LX * C::LY * (unsigned)sizeof(T));
-        tma_load_3d(ring0 + slot * C::PLANE, &tmap, &full_in[slot], X0, Y0, pin0 + j);
+        stage_plane_cp_async<T, C::LX, C::LY, 32>(ring0 + slot * C::PLANE, in, g, X0, Y0, pin0 + j, tid);
+        cp_async_mbar_arrive(&full_in[slot]);
       }
     }
     return;

@@ -106,6 +106,28 @@ __global__ void k_p2p_wait(const unsigned* a, const unsigned* b, unsigned v) {
   if (b) while ((int)(ld_acquire_sys(b) - v) < 0) __nanosleep(128);
 }
 
+// FMA throughput probe: the measured denominator of the "alu" roofline of
+// FMA-bound stencils (the paper lists each GPU's FP64 peak,
+// P:L222-L225). Every thread runs NACC independent fma chains x <- x*a + b for
+// iters x 8 steps (|a| < 1 keeps them bounded); the conditional store keeps the
+// chains live. FMAs per launch = blocks * 256 * iters * 8 * NACC.
+template <class T, int NACC>
+__global__ void __launch_bounds__(256) k_fma_probe(T* sink, long long iters, T a, T b) {
+  T x[NACC];
+#pragma unroll
+  for (int k = 0; k < NACC; ++k) x[k] = T(threadIdx.x + k) * T(1e-3);
+  for (long long i = 0; i < iters; ++i) {
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+#pragma unroll
+      for (int k = 0; k < NACC; ++k) x[k] = fma(x[k], a, b);
+  }
+  T s = T(0);
+#pragma unroll
+  for (int k = 0; k < NACC; ++k) s += x[k];
+  if (s == T(-12345)) sink[0] = s;
+}
+
 int grid_for(long long n) {
   long long b = (n + 255) / 256;
   const long long cap = 148LL * 16;
@@ -160,6 +182,22 @@ int launch_p2p_wait(const uint32_t* a, const uint32_t* b, uint32_t v, cudaStream
   k_p2p_wait<<<1, 1, 0, s>>>(a, b, v);
   g_launches.fetch_add(1);
   SM_CUDA(cudaGetLastError());
+  return STENCIL_OK;
+}
+
+int launch_fma_probe(int dtype, long long iters, int blocks_per_sm, void* sink, double* flops, cudaStream_t s) {
+  int dev = 0, nsm = 0;
+  SM_CUDA(cudaGetDevice(&dev));
+  SM_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
+  const int blocks = nsm * blocks_per_sm;
+  constexpr int NACC = 8;
+  if (dtype == STENCIL_F64)
+    k_fma_probe<double, NACC><<<blocks, 256, 0, s>>>((double*)sink, iters, 0.9990234375, 0.0009765625);
+  else
+    k_fma_probe<float, NACC><<<blocks, 256, 0, s>>>((float*)sink, iters, 0.9990234375f, 0.0009765625f);
+  g_launches.fetch_add(1);
+  SM_CUDA(cudaGetLastError());
+  *flops = 2.0 * blocks * 256.0 * (double)iters * 8.0 * NACC;
   return STENCIL_OK;
 }
 

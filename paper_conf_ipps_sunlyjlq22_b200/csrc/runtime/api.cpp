@@ -366,9 +366,8 @@ static int resolve_variant(stencil_plan_s* P) {
     const char* notma = getenv("STENCIL_NO_TMA");   // dev / test override: cp.async staging
     v.tma = rows_ok && b.lx <= 256 && b.ly <= 256 && b.lz <= 256 && !(notma && atoi(notma));
   }
-  if (fam == FAM_STREAM_TB && !v.tma)
-    SM_FAIL(STENCIL_E_OC_INFEASIBLE, "OC %s needs TMA staging (rows of 16-byte multiples, box <= 256)",
-            oc_name_static(P->oc));
+  // (streaming TB without TMA: the input planes are staged with element-wise
+  // cp.async -- rows that are not 16-byte multiples, boxes wider than 256)
   if (fam == FAM_STREAM_TB && v.tt < 2) v.family = FAM_STREAM;
   v.chunk = p.stream_chunk;
   v.sy = P->vdims[2];                       // = make_grid's strides (contiguous view)
@@ -593,7 +592,7 @@ static int get_tb_rem_kernel(stencil_plan_s* P, int tt, Variant* vout, Kernel* k
     v.ws_threads = v.tbrt_threads(P->pat, elem);
     if (v.ws_threads > 1024) SM_FAIL(STENCIL_E_OC_INFEASIBLE, "TB remainder CTA of %d threads", v.ws_threads);
   }
-  if (v.family == FAM_TILED && v.tma) {
+  if ((v.family == FAM_TILED || v.family == FAM_STREAM_TB) && v.tma) {
     const TmaBox b = tma_box(v, P->pat, elem);
     v.tma = b.lx <= 256 && b.ly <= 256 && b.lz <= 256;
   }
@@ -1103,17 +1102,23 @@ int stencil_plan_create(stencil_plan_t* plan, int ndim, const int64_t* dims, int
       P->params.bx /= 2;
     }
   }
+  std::string first_err;   // the reason at the requested (or default) setting
   for (int attempt = 0;; ++attempt) {
     const int rc = resolve_variant(P.get());
-    if (rc != STENCIL_E_OC_INFEASIBLE || attempt > 12) {
-      if (rc != STENCIL_OK) return rc;
-      break;
-    }
-    stencil_params_t& q = P->params;
-    if (!user_bz && q.bz > 1) q.bz /= 2;
-    else if (!user_by && q.by > 1 && (q.bx / std::max(q.vx, 1)) * (q.by / 2) >= 32) q.by /= 2;
-    else if (!user_bx && q.bx > 8 * q.vx) q.bx /= 2;
-    else return rc;
+    if (rc == STENCIL_E_OC_INFEASIBLE && first_err.empty()) first_err = t_err;
+    const bool give_up = [&] {
+      if (rc != STENCIL_E_OC_INFEASIBLE || attempt > 12) return true;
+      stencil_params_t& q = P->params;
+      if (!user_bz && q.bz > 1) q.bz /= 2;
+      else if (!user_by && q.by > 1 && (q.bx / std::max(q.vx, 1)) * (q.by / 2) >= 32) q.by /= 2;
+      else if (!user_bx && q.bx > 8 * q.vx) q.bx /= 2;
+      else return true;
+      return false;
+    }();
+    if (!give_up) continue;
+    if (rc == STENCIL_E_OC_INFEASIBLE) SM_FAIL(rc, "%s (no smaller default tile fits either)", first_err.c_str());
+    if (rc != STENCIL_OK) return rc;
+    break;
   }
   clear_error();
   if (P->var.reg_lo > 0 && !getenv("STENCIL_REGSPLIT")) {
@@ -1293,6 +1298,15 @@ int stencil_fill_field(void* dev, stencil_dtype_t dtype, int ndim, const int64_t
       SM_FAIL(STENCIL_E_INVAL, "box outside the global grid on axis %d", k);
   }
   return launch_fill(dev, dtype, b, o, g, seed, kind, (cudaStream_t)stream);
+}
+
+int stencil_fma_probe(stencil_dtype_t dtype, int64_t iters, int blocks_per_sm, void* sink, void* stream,
+                      double* flops) {
+  clear_error();
+  if (!sink || !flops) SM_FAIL(STENCIL_E_INVAL, "null argument");
+  if (dtype != STENCIL_F32 && dtype != STENCIL_F64) SM_FAIL(STENCIL_E_INVAL, "bad dtype");
+  if (iters < 1 || blocks_per_sm < 1 || blocks_per_sm > 8) SM_FAIL(STENCIL_E_INVAL, "iters >= 1, blocks_per_sm in 1..8");
+  return launch_fma_probe(dtype, iters, blocks_per_sm, sink, flops, (cudaStream_t)stream);
 }
 
 int stencil_slab_range(int64_t nz_global, int rank, int nranks, int64_t* z_begin, int64_t* z_end) {

@@ -397,6 +397,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   o << "  static constexpr int TMID = " << tmid << ";\n";
   o << "  static constexpr int MVX = " << (v.midvx > 0 ? v.midvx : std::max(v.vx, 1)) << ";\n";
   o << "  static constexpr bool SPLITMID = " << (v.splitmid ? "true" : "false") << ";\n";
+  o << "  static constexpr bool TMA = " << (v.tma ? "true" : "false") << ";   // streaming TB staging (else cp.async)\n";
   o << "  static constexpr bool XSHIFT = " << (v.xshift ? "true" : "false") << ";\n";
   o << "  static constexpr int XSH = " << (v.xshift ? pat.xlo % std::max(v.vx, 1) : 0) << ";\n";
   o << "  static constexpr int REG_LO = " << v.reg_lo << ", REG_HI = " << v.reg_hi << ";\n";

@@ -213,8 +213,87 @@ def random_coeffs(access: np.ndarray, seed: int) -> np.ndarray:
     return c / c.sum()
 
 
+# --------------------------------------------------------------------------
+# edge-case patterns (parity coverage of the method's degenerate cases)
+# --------------------------------------------------------------------------
+
+def pattern(ndim: int, order: int, weights: Dict[Tuple[int, ...], int], denom: int):
+    """Access tensor + dyadic coefficients ``weights[o] / denom`` for the
+    offsets ``o`` (slowest axis first). ``order`` is the DECLARED order (tensor
+    size 2r+1, frame width r); the offsets may reach less far (Table II
+    "order: the maximum extent", vs. the declared order of the
+    tensor). The centre is always accessed; its weight may be 0."""
+    acc, c = _empty(ndim, order)
+    ctr = (order,) * ndim
+    acc[ctr] = 1
+    for o, w in weights.items():
+        assert len(o) == ndim and max(abs(v) for v in o) <= order
+        idx = tuple(order + v for v in o)
+        acc[idx] = 1
+        c[idx] = w / float(denom)
+    return acc, c
+
+
+# One-sided / asymmetric extents, extent < declared order, no neighbours along
+# the streaming axis (NZ = 1), centre only, centre coefficient 0, mixed signs.
+# Positive patterns sum to <= 1 (outputs stay in (0, 2) for u0 in [1, 2), so the
+# pointwise relative error is well conditioned); the mixed-sign ones have
+# sum |c| <= 1 with denominators 2^4 -> exact for integer inputs up to 10 steps
+# in fp64 (10 + 4*10 <= 53, pin P7) and 3 steps in fp32 (10 + 4*3 <= 24).
+EDGE_3D: Dict[str, Tuple[int, Dict[Tuple[int, int, int], int], int]] = {
+    # zlo = 0, zhi = 2; ylo = 2, yhi = 1; xlo = 1, xhi = 3 (declared order 3)
+    "asym3d": (3, {(0, 0, 0): 6, (1, 0, 0): 3, (2, 0, 0): 2, (0, 0, -1): 3, (0, 0, 1): 2, (0, 0, 2): 2,
+                   (0, 0, 3): 1, (0, -2, 0): 2, (0, -1, 1): 3, (0, 1, 0): 2, (1, 1, 3): 1, (2, -2, -1): 1,
+                   (1, -1, 2): 4}, 32),
+    # mirror: zlo = 3, zhi = 0; ylo = 0, yhi = 2; xlo = 3, xhi = 0
+    "asym3d_lo": (3, {(0, 0, 0): 8, (-1, 0, 0): 4, (-3, 0, 0): 2, (0, 0, -3): 2, (0, 0, -1): 4, (0, 2, 0): 4,
+                      (0, 1, -2): 4, (-2, 1, -1): 2, (-1, 2, -3): 2}, 32),
+    # extent 1 (the heat star) declared as order 3: frame width 3, halo 1
+    "ext_lt_order3d": (3, {(0, 0, 0): 2, (1, 0, 0): 1, (-1, 0, 0): 1, (0, 1, 0): 1, (0, -1, 0): 1,
+                           (0, 0, 1): 1, (0, 0, -1): 1}, 8),
+    # no z neighbours (NZ = 1 plane in the streaming window): in-plane order 2
+    "flat3d": (2, {(0, 0, 0): 4, (0, 0, 1): 2, (0, 0, -1): 2, (0, 1, 0): 2, (0, -1, 0): 2, (0, 1, 1): 1,
+                   (0, -1, -1): 1, (0, 2, 0): 1, (0, 0, -2): 1}, 16),
+    # z neighbours only (no in-plane halo)
+    "zonly3d": (2, {(0, 0, 0): 4, (1, 0, 0): 1, (-1, 0, 0): 1, (2, 0, 0): 1, (-2, 0, 0): 1}, 8),
+    # centre only; centre coefficient 0 (heat arms only)
+    "centre3d": (1, {(0, 0, 0): 1}, 2),
+    "zero_centre3d": (1, {(0, 0, 0): 0, (1, 0, 0): 1, (-1, 0, 0): 1, (0, 1, 0): 1, (0, -1, 0): 1,
+                          (0, 0, 1): 1, (0, 0, -1): 1}, 8),
+    # mixed signs, sum |k| = 16 = 2^4
+    "mixed3d": (1, {(0, 0, 0): 5, (1, 0, 0): -2, (-1, 0, 0): 1, (0, 1, 0): 2, (0, -1, 1): -1, (0, 0, -1): 3,
+                    (1, 1, 1): -1, (-1, -1, 0): 1}, 16),
+    "mixed3d_r2": (2, {(0, 0, 0): 4, (2, 0, 0): -1, (-1, 0, 0): 2, (0, -2, 1): -2, (0, 1, 0): 1, (0, 0, 2): 3,
+                       (1, 2, -2): -1, (-2, -1, -1): 2}, 16),
+}
+EDGE_2D: Dict[str, Tuple[int, Dict[Tuple[int, int], int], int]] = {
+    # ylo = 0, yhi = 2; xlo = 1, xhi = 3
+    "asym2d": (3, {(0, 0): 6, (1, 0): 3, (2, 0): 2, (0, -1): 3, (0, 1): 2, (0, 3): 2, (1, 2): 1, (2, -1): 1,
+                   (1, -1): 2}, 22 + 10),
+    "asym2d_lo": (2, {(0, 0): 4, (-2, 0): 2, (-1, -2): 1, (0, -1): 1}, 8),
+    "ext_lt_order2d": (2, {(0, 0): 4, (1, 0): 1, (-1, 0): 1, (0, 1): 1, (0, -1): 1}, 8),
+    # x neighbours only: NZ = 1 row in the streaming (y) window
+    "row2d": (3, {(0, 0): 4, (0, -3): 1, (0, -1): 1, (0, 1): 1, (0, 2): 1}, 8),
+    # y neighbours only (no x halo)
+    "col2d": (2, {(0, 0): 4, (1, 0): 1, (-1, 0): 1, (2, 0): 1, (-2, 0): 1}, 8),
+    "centre2d": (1, {(0, 0): 1}, 2),
+    "zero_centre2d": (1, {(0, 0): 0, (1, 0): 1, (-1, 0): 1, (0, 1): 1, (0, -1): 1}, 4),
+    "mixed2d": (2, {(0, 0): 5, (1, 0): -2, (-2, 0): 1, (0, 1): 2, (1, -2): -1, (0, -1): 3, (-1, 2): -2}, 16),
+}
+
+
+def edge_stencil(name: str):
+    if name in EDGE_3D:
+        r, w, d = EDGE_3D[name]
+        return pattern(3, r, w, d)
+    r, w, d = EDGE_2D[name]
+    return pattern(2, r, w, d)
+
+
 def config_stencil(name: str, seed: int = 0):
     """Named workloads of BASELINE.json configs."""
+    if name.startswith("edge:"):
+        return edge_stencil(name[5:])
     if name == "heat2d":
         return heat2d()
     if name == "heat3d":
