@@ -11,6 +11,7 @@ C-ABI schedule on one GPU through the loopback transport.
   the gathered result must equal the single-plan run bitwise (P10).
 """
 import os
+import socket
 
 import numpy as np
 import pytest
@@ -77,16 +78,30 @@ def _worker(rank, world, port, name, gdims, steps, T, result_q):
 
 
 @pytest.mark.parametrize("world,name,steps,T", [(2, "heat3d", 5, 1), (3, "random3d:2:5", 4, 2),
-                                                (2, "random3d:1:3", 6, 4)])
+                                                (2, "random3d:1:3", 6, 4),
+                                                # one-sided / asymmetric z extents (declared order 3)
+                                                (2, "edge:asym3d", 5, 2), (3, "edge:asym3d_lo", 4, 1)])
 def test_gloo_slab_exchange_matches_oracle(world, name, steps, T):
-    gdims = (60, 12, 14)
+    gdims = (60, 12, 14) if not name.startswith("edge:") else (84, 12, 14)
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    port = 29500 + world * 7 + steps
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
     procs = [ctx.Process(target=_worker, args=(k, world, port, name, gdims, steps, T, q)) for k in range(world)]
     for p in procs:
         p.start()
-    got = q.get(timeout=300)
+    import queue
+    import time
+    t_end = time.time() + 300
+    while True:          # fail fast when a rank dies instead of waiting out the timeout
+        try:
+            got = q.get(timeout=2)
+            break
+        except queue.Empty:
+            dead = [p.exitcode for p in procs if p.exitcode not in (None, 0)]
+            assert not dead and time.time() < t_end, f"gloo ranks failed: exit codes {dead}"
     for p in procs:
         p.join(timeout=60)
         assert p.exitcode == 0
@@ -136,7 +151,10 @@ def _loopback(name, gdims, dtype, oc, steps, P, params=None):
 @pytest.mark.parametrize("name,dtype,oc,steps,P", [
     ("heat3d", "f64", "base", 3, 2), ("heat3d", "f64", "ST_RT_PR", 4, 3), ("random3d:2:5", "f64", "TB", 5, 2),
     ("random3d:3:1", "f32", "ST_TB_RT_PR", 5, 3), ("star25", "f32", "ST_BM_PR", 3, 2),
-    ("box125", "f64", "ST_TB_CM", 4, 2)])
+    ("box125", "f64", "ST_TB_CM", 4, 2),
+    # one-sided / asymmetric z extents: halo counts differ per side (C-18)
+    ("edge:asym3d", "f64", "ST_TB_RT_PR", 5, 3), ("edge:asym3d_lo", "f64", "ST_BM_RT_PR", 4, 2),
+    ("edge:zonly3d", "f32", "TB", 5, 2), ("edge:flat3d", "f64", "ST_TB_CM", 4, 2)])
 def test_loopback_slabs_bitwise(gpu, name, dtype, oc, steps, P):
     gdims = (100, 36, 48)
     got, ref, full = _loopback(name, gdims, dtype, oc, steps, P)

@@ -44,7 +44,12 @@ def _slab_input(full, z0, z1, G, shape):
     ("random3d:3:1", "f32", "ST_TB_RT_PR", 4, 3, {"tb_steps": 3}),
     ("star25", "f32", "ST_BM_PR", 3, 2, None),
     ("box125", "f64", "ST_TB_CM", 4, 2, None),
-    ("random3d:1:2", "f64", "ST_CM_RT", 6, 4, None)])
+    ("random3d:1:2", "f64", "ST_CM_RT", 6, 4, None),
+    # one-sided / asymmetric z extents: the mirrored plane ranges differ per side
+    ("edge:asym3d", "f64", "ST_TB_BM_RT_PR", 5, 3, None),       # zlo = 0, zhi = 2
+    ("edge:asym3d_lo", "f64", "ST_RT_PR", 4, 2, None),          # zlo = 3, zhi = 0
+    ("edge:zonly3d", "f32", "ST_TB_RT_PR", 5, 2, None),
+    ("edge:asym3d", "f64", "TB_CM", 6, 2, {"tb_steps": 3})])
 def test_p2p_in_process_bitwise(gpu, name, dtype, oc, steps, P, params):
     acc, c = si.config_stencil(name)
     gdims = (96, 36, 48) if P <= 3 else (160, 30, 40)
@@ -154,7 +159,8 @@ def _free_port():
 
 
 @pytest.mark.parametrize("name,dtype,oc,steps", [("heat3d", "f64", "ST_TB_BM_RT_PR", 5),
-                                                  ("random3d:2:5", "f64", "ST_RT_PR", 4)])
+                                                  ("random3d:2:5", "f64", "ST_RT_PR", 4),
+                                                  ("edge:asym3d", "f64", "ST_TB_CM_RT_PR", 5)])
 def test_p2p_two_processes_ipc(gpu, tmp_path, name, dtype, oc, steps):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
