@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-#define STENCIL_ABI_VERSION 1
+#define STENCIL_ABI_VERSION 2
 
 /* Opaque plan: one stencil on one grid shape under one OC and parameter
  * setting. Created by stencil_plan_create, owned by the caller, released by
@@ -190,7 +190,11 @@ int stencil_run_host(stencil_plan_t plan, const void *in_host, void *out_host, i
  * settings. Infeasible OCs get +INF. best_oc = argmin over finite times, ties
  * to the smallest id. With a communicator, per-OC times are the max over ranks
  * (all ranks return identical vectors). `in` is preserved, `out` receives the
- * last run's result. Outputs:
+ * last run's result. Error containment: a setting whose plan is infeasible
+ * (E_OC_INFEASIBLE) or whose launch fails while the CUDA context stays usable
+ * counts as a crash of that setting (+INF, the row's status says why) and the
+ * sweep goes on; E_INVAL from a sampled setting (a sampler bug), a sticky CUDA
+ * error, an NCCL error or an NVRTC failure fails the whole call. Outputs:
  *   times_ms[30], oc_ids[30] (ascending), best_params[30], *best_oc.
  * Synchronises the plan's stream. */
 int stencil_oc_sweep(stencil_plan_t plan, const void *in_dev, void *out_dev, int steps,
@@ -244,12 +248,17 @@ int stencil_embed_tensor(int ndim, int order, const uint8_t *access, uint8_t *ou
  * "each parameter setting and its corresponding execution time are also
  * stored"): one row per (OC, setting) tried, in sweep order. Writes at
  * most max_rows rows and the total count to *nrows. time_ms = +INF if the
- * setting was infeasible. */
+ * setting did not run; `status` says why: STENCIL_OK (timed),
+ * STENCIL_E_OC_INFEASIBLE (a resource limit: the paper's "crash"), or
+ * the code of a launch error that left the CUDA context usable (contained to
+ * this setting; see stencil_oc_sweep). */
 typedef struct {
     uint32_t oc;
     int32_t setting;          /* k of stencil_sample_params */
-    stencil_params_t params;  /* resolved setting (defaults filled in) */
+    stencil_params_t params;  /* resolved setting (defaults filled in; the raw
+                                 sample when the plan could not be created) */
     float time_ms;            /* median of the timed runs */
+    int32_t status;           /* STENCIL_OK or the reason time_ms is +INF */
 } stencil_sweep_row_t;
 
 int stencil_sweep_rows(stencil_plan_t plan, stencil_sweep_row_t *rows, int max_rows, int *nrows);

@@ -70,7 +70,7 @@ class Features(ctypes.Structure):
 
 class SweepRow(ctypes.Structure):
     _fields_ = [("oc", ctypes.c_uint32), ("setting", ctypes.c_int32), ("params", Params),
-                ("time_ms", ctypes.c_float)]
+                ("time_ms", ctypes.c_float), ("status", ctypes.c_int32)]
 
 
 class P2PBuffers(ctypes.Structure):
@@ -440,8 +440,29 @@ class Plan:
         _check(L.stencil_run(self._h, ctypes.c_void_p(inp.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                              int(steps)))
 
+    def _check_host(self, a, name):
+        """A host buffer for stencil_run_host: C-contiguous, the plan's dtype and
+        array_shape, exactly workspace_bytes() long (the C call copies that many
+        bytes each way, so anything smaller would be overrun)."""
+        shape = self.array_shape
+        want = np.float64 if self.dtype == F64 else np.float32
+        if hasattr(a, "data_ptr"):            # torch
+            ok = (not a.is_cuda and a.is_contiguous() and a.dtype == self.torch_dtype and tuple(a.shape) == shape
+                  and a.numel() * a.element_size() == self.workspace_bytes())
+        else:
+            a = np.asarray(a) if not isinstance(a, np.ndarray) else a
+            ok = (a.flags.c_contiguous and a.dtype == want and tuple(a.shape) == shape
+                  and a.nbytes == self.workspace_bytes())
+        if not ok:
+            raise ValueError(f"{name}: expected a C-contiguous host {want.__name__} buffer of shape {shape}")
+        if name == "out" and not hasattr(a, "data_ptr") and not a.flags.writeable:
+            raise ValueError("out: host buffer is read-only")
+
     def run_host(self, inp, out, steps: int, stream=None) -> None:
         """End to end: host buffers in and out (pinned torch tensors or numpy)."""
+        self._check_host(inp, "in")
+        self._check_host(out, "out")
+
         def ptr(a):
             return a.data_ptr() if hasattr(a, "data_ptr") else a.ctypes.data
         L = lib()
@@ -472,7 +493,8 @@ class Plan:
             "best_params": [bp[i].to_dict() for i in range(NUM_OC)],
             "best_oc": int(best.value),
             "rows": [{"oc": int(r.oc), "oc_name": oc_name(r.oc), "setting": int(r.setting),
-                      "params": r.params.to_dict(), "time_ms": float(r.time_ms)} for r in rows[:n.value]],
+                      "params": r.params.to_dict(), "time_ms": float(r.time_ms), "status": int(r.status)}
+                     for r in rows[:n.value]],
         }
 
     def set_timing(self, enable: bool) -> None:

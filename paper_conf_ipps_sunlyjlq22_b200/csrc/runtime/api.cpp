@@ -926,6 +926,18 @@ static int run_host_pipelined(stencil_plan_s* P, const void* hin, void* hout, in
     P->h2d_ev.push_back(a);
     P->cmp_ev.push_back(b);
   }
+  // On an error return, copies already queued still read / write the caller's
+  // host buffers: drain every stream before handing control back.
+  struct Drain {
+    stencil_plan_s* P;
+    bool armed = true;
+    ~Drain() {
+      if (!armed) return;
+      cudaStreamSynchronize(P->h2d_stream);
+      cudaStreamSynchronize(P->d2h_stream);
+      cudaStreamSynchronize(P->stream);
+    }
+  } drain{P};
   // the copy streams start after everything queued on the plan's stream
   SM_CUDA(cudaEventRecord(P->cmp_ev[0], P->stream));
   SM_CUDA(cudaStreamWaitEvent(P->h2d_stream, P->cmp_ev[0], 0));
@@ -984,9 +996,19 @@ static int run_host_pipelined(stencil_plan_s* P, const void* hin, void* hout, in
   SM_CUDA(cudaGetLastError());
   SM_CUDA(cudaStreamSynchronize(P->d2h_stream));
   SM_CUDA(cudaStreamSynchronize(P->stream));
+  drain.armed = false;
   P->host_chunks = K;
   *done = true;
   return STENCIL_OK;
+}
+
+void free_host_path_buffers(stencil_plan_s* P) {
+  if (P->h_in_dev || P->h_out_dev || P->h_ws_dev) cudaDeviceSynchronize();   // no copy may still use them
+  if (P->h_in_dev) cudaFree(P->h_in_dev);
+  if (P->h_out_dev) cudaFree(P->h_out_dev);
+  if (P->h_ws_dev) cudaFree(P->h_ws_dev);
+  P->h_in_dev = P->h_out_dev = P->h_ws_dev = nullptr;
+  P->h_bytes = 0;
 }
 
 int run_device(stencil_plan_s* P, const void* in, void* out, int steps) {
@@ -1251,12 +1273,16 @@ int stencil_run(stencil_plan_t plan, const void* in, void* out, int steps) {
 int stencil_run_host(stencil_plan_t P, const void* in_host, void* out_host, int steps) {
   clear_error();
   if (!P || !in_host || !out_host) SM_FAIL(STENCIL_E_INVAL, "null argument");
+  if (P->comm && P->comm->transport == TR_P2P)
+    SM_FAIL(STENCIL_E_STATE, "P2P slab plans run only on their registered device buffers");
   const size_t bytes = stencil_plan_workspace_bytes(P);
+  if (P->h_bytes < bytes) free_host_path_buffers(P);   // the view grew (slab ghosts): reallocate
   if (!P->h_in_dev) SM_CUDA(cudaMalloc(&P->h_in_dev, bytes));
   if (!P->h_out_dev) SM_CUDA(cudaMalloc(&P->h_out_dev, bytes));
+  P->h_bytes = bytes;
   void* saved_ws = P->ws;
   size_t saved_b = P->ws_bytes;
-  if (!P->ws) {
+  if (!P->ws || P->ws_bytes < bytes) {
     if (!P->h_ws_dev) SM_CUDA(cudaMalloc(&P->h_ws_dev, bytes));
     P->ws = P->h_ws_dev;
     P->ws_bytes = bytes;

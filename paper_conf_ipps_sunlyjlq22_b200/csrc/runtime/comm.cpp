@@ -22,6 +22,7 @@ void comm_destroy(Comm* c) {
   if (c->ev_comm) cudaEventDestroy(c->ev_comm);
   if (c->edge_stream) cudaStreamDestroy(c->edge_stream);
   if (c->ev_main) cudaEventDestroy(c->ev_main);
+  if (c->red_buf) cudaFree(c->red_buf);
   delete c;
 }
 
@@ -50,8 +51,21 @@ void slab_halo(int G, int n, int zlo_g, int zhi_g, int rank, int nranks, int64_t
   out[6] = G + n;      out[7] = hi ? zhi_g : 0;
 }
 
+// A failed peer or network error surfaces asynchronously in NCCL: check the
+// communicator before every exchange and after the label all-reduce.
+int comm_check_async(const Comm* c) {
+  if (!c || c->transport != TR_NCCL || !c->nccl) return STENCIL_OK;
+  ncclResult_t ar = ncclSuccess;
+  const ncclResult_t r = ncclCommGetAsyncError((ncclComm_t)c->nccl, &ar);
+  if (r != ncclSuccess) SM_FAIL(STENCIL_E_NCCL, "ncclCommGetAsyncError: %s", ncclGetErrorString(r));
+  if (ar != ncclSuccess && ar != ncclInProgress)
+    SM_FAIL(STENCIL_E_NCCL, "NCCL communicator failed asynchronously: %s", ncclGetErrorString(ar));
+  return STENCIL_OK;
+}
+
 int comm_exchange_nccl(stencil_plan_s* P, void* buf, int tl) {
   Comm* c = P->comm;
+  SM_TRY(comm_check_async(c));
   const int elem = P->dtype == STENCIL_F64 ? 8 : 4;
   const size_t plane = (size_t)P->vdims[1] * P->vdims[2];
   int64_t h[8];
@@ -87,18 +101,18 @@ int comm_attach(stencil_plan_s* child, const stencil_plan_s* parent) {
 }
 
 int comm_allreduce_max(stencil_plan_s* P, float* v, int n) {
-  if (P->comm->transport != TR_NCCL) return STENCIL_OK;
-  float* d = nullptr;
-  SM_CUDA(cudaMalloc(&d, sizeof(float) * n));
+  Comm* c = P->comm;
+  if (c->transport != TR_NCCL) return STENCIL_OK;
+  if (n < 1 || n > 64) SM_FAIL(STENCIL_E_INVAL, "all-reduce of %d values", n);
+  SM_TRY(comm_check_async(c));
+  if (!c->red_buf) SM_CUDA(cudaMalloc(&c->red_buf, sizeof(float) * 64));   // once per communicator
+  float* d = c->red_buf;
   SM_CUDA(cudaMemcpyAsync(d, v, sizeof(float) * n, cudaMemcpyHostToDevice, P->stream));
-  ncclResult_t r = ncclAllReduce(d, d, n, ncclFloat32, ncclMax, (ncclComm_t)P->comm->nccl, P->stream);
-  if (r != ncclSuccess) {
-    cudaFree(d);
-    SM_FAIL(STENCIL_E_NCCL, "ncclAllReduce: %s", ncclGetErrorString(r));
-  }
+  ncclResult_t r = ncclAllReduce(d, d, n, ncclFloat32, ncclMax, (ncclComm_t)c->nccl, P->stream);
+  if (r != ncclSuccess) SM_FAIL(STENCIL_E_NCCL, "ncclAllReduce: %s", ncclGetErrorString(r));
   SM_CUDA(cudaMemcpyAsync(v, d, sizeof(float) * n, cudaMemcpyDeviceToHost, P->stream));
   SM_CUDA(cudaStreamSynchronize(P->stream));
-  cudaFree(d);
+  SM_TRY(comm_check_async(c));
   return STENCIL_OK;
 }
 
@@ -127,6 +141,7 @@ static int slab_setup(stencil_plan_s* P, int rank, int nranks, int transport) {
   P->ghost = G;
   P->vdims[0] = P->dims[0] + 2 * G;
   P->tmaps.clear();
+  free_host_path_buffers(P);   // stencil_run_host sized them for the old view
   return STENCIL_OK;
 }
 

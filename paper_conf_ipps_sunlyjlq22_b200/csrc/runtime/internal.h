@@ -149,6 +149,7 @@ struct Comm {
   cudaEvent_t ev_comm = nullptr;     // halo exchange into dst done (comm stream)
   cudaStream_t edge_stream = nullptr;  // high-priority stream of the edge-plane kernels
   cudaEvent_t ev_main = nullptr;     // main stream reached the edge launch (previous interior done)
+  float* red_buf = nullptr;          // device buffer of the label all-reduce (64 floats, owned)
   std::vector<stencil_plan_s*> peers;  // LOOPBACK: plans of all ranks (index = rank)
   const void* cur = nullptr;         // LOOPBACK: buffer this rank is exchanging (for peers)
   // P2P (fused halo): registered grids of this rank and its neighbours
@@ -166,6 +167,8 @@ int comm_create_stream_events(Comm* c);
 void slab_halo(int ghost, int n, int zlo_g, int zhi_g, int rank, int nranks, int64_t out[8]);
 int comm_exchange_nccl(stencil_plan_s* P, void* buf, int tl);
 int comm_allreduce_max(stencil_plan_s* P, float* v, int n);
+int comm_check_async(const Comm* c);   // asynchronous NCCL errors (ncclCommGetAsyncError)
+void free_host_path_buffers(stencil_plan_s* P);
 
 // ---------------------------------------------------------------- plan
 struct stencil_plan_impl;
@@ -207,6 +210,7 @@ struct stencil_plan_s {
   void* h_in_dev = nullptr;
   void* h_out_dev = nullptr;
   void* h_ws_dev = nullptr;
+  size_t h_bytes = 0;                // size of each of the three host-path buffers
   cudaStream_t h2d_stream = nullptr, d2h_stream = nullptr;   // pipelined stencil_run_host
   std::vector<cudaEvent_t> h2d_ev, cmp_ev;
   int host_chunks = 0;           // chunks of the last stencil_run_host (0 = not pipelined)

@@ -6,7 +6,9 @@ setting and its corresponding execution time are also stored in the stencil
 dataset" (§IV-A). One JSON line per (stencil, OC, setting) plus one
 label line per stencil; features come from the Table II extractor and the 9^d
 tensor of Fig. 6 (both in libstencilmart.so). Files are append-only JSONL, so an
-interrupted run resumes by skipping stencil ids already labelled.
+interrupted run resumes by skipping stencil ids already labelled (`resume`
+first cuts a torn tail: a partial last line and the setting rows of a stencil
+whose label line was never written).
 """
 from __future__ import annotations
 
@@ -34,6 +36,37 @@ def done_ids(path: str) -> Set[str]:
     return out
 
 
+def resume(path: str) -> Set[str]:
+    """Make an interrupted dataset file appendable and return the labelled ids.
+
+    A stencil's rows are appended as one block ending with its label line, so
+    everything after the last complete label line -- a torn last line, or the
+    setting rows of a stencil whose label never landed -- belongs to a stencil
+    that must be swept again: the file is truncated there (it would otherwise
+    leave duplicate setting rows, or glue the next row onto the torn line)."""
+    if not os.path.exists(path):
+        return set()
+    keep = 0
+    out: Set[str] = set()
+    with open(path, "rb") as f:
+        pos = 0
+        for raw in f:
+            pos += len(raw)
+            if not raw.endswith(b"\n"):
+                break                             # torn last line
+            try:
+                d = json.loads(raw)
+            except json.JSONDecodeError:
+                break
+            if d.get("kind") == "label":
+                out.add(d["stencil_id"])
+                keep = pos
+    if keep != os.path.getsize(path):
+        with open(path, "r+b") as f:
+            f.truncate(keep)
+    return out
+
+
 def label_stencil(stencil_id: str, access: np.ndarray, coeffs: np.ndarray, dims: Sequence[int], dtype: str,
                   steps: int = 4, settings_per_oc: int = 4, reps: int = 3, seed: int = 0,
                   field_seed: int = 1) -> List[dict]:
@@ -53,7 +86,7 @@ def label_stencil(stencil_id: str, access: np.ndarray, coeffs: np.ndarray, dims:
     for r in res["rows"]:
         t = r["time_ms"]
         rows.append(dict(common, kind="setting", oc=r["oc"], oc_name=r["oc_name"], setting=r["setting"],
-                         params=r["params"], time_ms=t if math.isfinite(t) else None))
+                         params=r["params"], time_ms=t if math.isfinite(t) else None, status=r["status"]))
     rows.append(dict(common, kind="label", best_oc=res["best_oc"], best_oc_name=oc_name(res["best_oc"]),
                      oc_times_ms={oc_name(o): (t if math.isfinite(t) else None)
                                   for o, t in zip(res["oc_ids"], res["times_ms"])},

@@ -24,7 +24,7 @@ ap.add_argument("--steps", type=int, default=4)
 ap.add_argument("--settings", type=int, default=3)
 ap.add_argument("--seed", type=int, default=0)
 a = ap.parse_args()
-done = dataset.done_ids(a.out)
+done = dataset.resume(a.out)      # cut a torn tail of an interrupted run
 for i in range(a.n):
     order = 1 + i % 4
     sid = f"{a.ndim}d-o{order}-s{a.seed + i}"

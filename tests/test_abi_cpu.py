@@ -30,7 +30,7 @@ def test_exports_every_header_symbol():
     for n in sorted(names):
         assert hasattr(L, n), n
     assert names == set(sm.exported_symbols())
-    assert L.stencil_abi_version() == 1
+    assert L.stencil_abi_version() == 2
 
 
 def test_oc_lattice_matches_oracle():

@@ -358,3 +358,64 @@ def test_tb_rt_interior_and_edge_tiles(gpu, name, dims, dtype, oc, prm):
     got = _run(sm.Plan(dims, acc, c, dtype, sm.oc_from_name(oc), prm), u0, dtype, steps)
     assert _relerr(got, ref) <= TOL[dtype]
     assert np.array_equal(got, base)
+
+
+def test_sweep_rows(gpu):
+    """NEXT-1: the label generator's rows (stencil_sweep_rows; "each
+    parameter setting and its corresponding execution time are also stored"):
+    30 x K rows in sweep order (OC ids ascending, settings 0..K-1); each row's
+    setting is the resolved stencil_sample_params(seed, oc, k) (k = 0: the
+    defaults), or the raw sample when the setting is infeasible; per OC the
+    label time is the minimum over its rows (bit-exact) and best_params the
+    first argmin row."""
+    torch = _torch()
+    acc, c = si.config_stencil("random3d:2:6")
+    dims, dtype, K, seed = (36, 40, 56), "f64", 3, 11
+    x = torch.empty(dims, dtype=torch.float64, device="cuda")
+    sm.fill_field(x, 4)
+    y = torch.empty_like(x)
+    res = sm.Plan(dims, acc, c, dtype, 0).oc_sweep(x, y, steps=2, settings_per_oc=K, reps=3, seed=seed)
+    rows = res["rows"]
+    ids = oracle.valid_ocs()
+    assert res["oc_ids"] == ids and len(rows) == len(ids) * K
+    for i, oc in enumerate(ids):
+        rr = rows[i * K:(i + 1) * K]
+        assert [r["oc"] for r in rr] == [oc] * K and [r["setting"] for r in rr] == list(range(K))
+        for k, r in enumerate(rr):
+            raw = sm.sample_params(oc, 3, dtype, seed, k)
+            if math.isfinite(r["time_ms"]):
+                want = sm.Plan(dims, acc, c, dtype, oc, None if k == 0 else raw).info["params"]
+            else:
+                want = raw
+            assert r["params"] == want, (sm.oc_name(oc), k)
+        ts = [r["time_ms"] for r in rr]
+        fin = [t for t in ts if math.isfinite(t)]
+        if not fin:
+            assert not math.isfinite(res["times_ms"][i])
+            continue
+        assert res["times_ms"][i] == min(fin), sm.oc_name(oc)
+        assert res["best_params"][i] == rr[ts.index(min(fin))]["params"], sm.oc_name(oc)
+    assert res["best_oc"] == oracle.best_oc(res["times_ms"], res["oc_ids"])
+
+
+@pytest.mark.parametrize("cfg,oc", [("C2", "ST_TB_BM_RT_PR"), ("C2", "ST_RT_PR"), ("C4", "ST_CM_RT_PR"),
+                                    ("C4", "ST_BM_RT_PR")])
+def test_full_grid_elementwise(gpu, cfg, oc):
+    """BASELINE sizes, whole grid, element by element against the oracle after
+    the config's 10 steps, with the default setting of the OC the bench labels
+    (C2: ST_TB_BM_RT_PR, C4: ST_CM_RT_PR) and the runner-up."""
+    torch = _torch()
+    C = si.CONFIGS[cfg]
+    acc, c = si.config_stencil(C["stencil"])
+    dims, dtype, steps = C["dims"], C["dtype"], C["steps"]
+    x = torch.empty(dims, dtype=torch.float64, device="cuda")
+    sm.fill_field(x, C["seed"])
+    y = torch.empty_like(x)
+    sm.Plan(dims, acc, c, dtype, sm.oc_from_name(oc)).run(x, y, steps)
+    torch.cuda.synchronize()
+    got = y.cpu().numpy()
+    del y
+    ref = oracle.sweep(x.cpu().numpy(), acc, c, steps, dtype=dtype)
+    del x
+    torch.cuda.empty_cache()
+    assert _relerr(got, ref) <= TOL[dtype], oc
