@@ -86,23 +86,19 @@ def performance(times: np.ndarray) -> np.ndarray:
 
 
 def pearson(x: Sequence[float], y: Sequence[float]) -> float:
-    """Textbook PCC: cov(x, y) / (sd(x) sd(y)); 0 if undefined (< 3 points or zero variance)."""
+    """Textbook PCC: cov(x, y) / (sd(x) sd(y)); 0 if undefined (< 3 points or zero variance).
+
+    Sums are exactly rounded (math.fsum): the oracle states the definition, it
+    does not mimic any summation order of the product (tests compare the PCC at
+    a tolerance and the groups only where the ranking is not a rounding tie)."""
     n = len(x)
     if n < 3:
         return 0.0
-    # plain left-to-right loops (Python's sum() of floats is compensated since 3.12)
-    mx = 0.0
-    my = 0.0
-    for a, b in zip(x, y):
-        mx += a
-        my += b
-    mx /= n
-    my /= n
-    sxy = sxx = syy = 0.0
-    for a, b in zip(x, y):
-        sxy += (a - mx) * (b - my)
-        sxx += (a - mx) * (a - mx)
-        syy += (b - my) * (b - my)
+    mx = math.fsum(x) / n
+    my = math.fsum(y) / n
+    sxy = math.fsum((a - mx) * (b - my) for a, b in zip(x, y))
+    sxx = math.fsum((a - mx) * (a - mx) for a in x)
+    syy = math.fsum((b - my) * (b - my) for b in y)
     if sxx == 0.0 or syy == 0.0:
         return 0.0
     return sxy / math.sqrt(sxx * syy)
@@ -139,11 +135,23 @@ def groups(times: np.ndarray, n_classes: int = 5) -> Tuple[List[int], List[int]]
     pairs ... can be grouped to reduce the classes to be predicted"; P:L234:
     "reduce the number of predicted OCs to 5").
     """
+    return groups_from_pcc(times, pcc(times), n_classes)
+
+
+def ranking_is_tie_free(p: np.ndarray, tol: float = 1e-9) -> bool:
+    """True when no two pairs' |PCC| differ by a rounding-level amount (0 < d <= tol):
+    then any PCC within tol/2 of these values ranks the pairs the same way."""
+    v = sorted(r[0] for r in ranked_pairs(p))
+    return all(not (0.0 < b - a <= tol) for a, b in zip(v, v[1:]))
+
+
+def groups_from_pcc(times: np.ndarray, p: np.ndarray, n_classes: int = 5) -> Tuple[List[int], List[int]]:
+    """The merge of :func:`groups` on a given PCC matrix `p`."""
     k = times.shape[1]
     member = [{j} for j in range(k)]          # plain sets, merged explicitly
     where = list(range(k))
     count = k
-    for _, a, b in ranked_pairs(pcc(times)):
+    for _, a, b in ranked_pairs(p):
         if count <= n_classes:
             break
         ga, gb = where[a], where[b]
