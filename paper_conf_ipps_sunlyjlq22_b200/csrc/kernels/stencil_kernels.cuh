@@ -81,6 +81,19 @@ __device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned
 __device__ __forceinline__ void mbar_arrive(unsigned long long* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
 }
+// One arrival per warp (S::ELECT barriers count warps, not threads): the warp's
+// shared-memory reads / writes are ordered before lane 0's release-arrive by
+// __syncwarp, so a waiter that acquires the phase sees all of them. 32 lanes
+// arriving on one mbarrier word are 32 shared-memory atomics; one is enough.
+template <bool ELECT>
+__device__ __forceinline__ void warp_arrive(unsigned long long* bar) {
+  if constexpr (ELECT) {
+    __syncwarp();
+    if ((threadIdx.x & 31) == 0) mbar_arrive(bar);
+  } else {
+    mbar_arrive(bar);
+  }
+}
 // wait with a suspend-time hint: the warp sleeps in the barrier unit instead of
 // spinning through issue slots (warp-specialised pipelines wait a lot)
 __device__ __forceinline__ void mbar_wait_sleep(unsigned long long* bar, unsigned parity) {
@@ -281,7 +294,7 @@ __device__ __forceinline__ void stage_plane_cp_async(T* dst, const T* in, const 
 // An op is either a window LOAD of VX consecutive values of one plane, or an
 // FMA of one loaded value into one accumulator:
 //   LOAD (bit31 = 0): zi = op & 15, row j = ((op >> 4) & 255) - 128,
-//                     vector kv = ((op >> 12) & 15) - 8  (columns [kv*VX, kv*VX+VX))
+//                     vector kv = ((op >> 12) & 4095) - 2048  (columns [kv*VX, kv*VX+VX))
 //   FMA  (bit31 = 1): coefficient id = op & 1023, element e = (op >> 10) & 3,
 //                     output column v = (op >> 12) & 3, output row m = (op >> 14) & 7,
 //                     slice zi = (op >> 17) & 15; bit 30 (fp32 only): packed pair,
@@ -303,7 +316,7 @@ __device__ __forceinline__ void run_gather_ops(const L (&pl)[S::NZ], typename S:
   for (int i = 0; i < O::NOPS; ++i) {
     const unsigned op = O::op(i);
     if (!(op >> 31)) {
-      pl[op & 15].get(int((op >> 4) & 255) - 128, int((op >> 12) & 15) - 8, w);
+      pl[op & 15].get(int((op >> 4) & 255) - 128, int((op >> 12) & 4095) - 2048, w);
     } else if (op & 0x40000000u) {
       T* a = &acc[(op >> 14) & 7][(op >> 12) & 3];
       fma2_t(S::coef(op & 1023), w[(op >> 10) & 3], w[((op >> 10) & 3) + 1], a[0], a[1]);
@@ -328,7 +341,7 @@ __device__ __forceinline__ void run_scatter_ops(const L& pl, typename S::T (&acc
   for (int i = 0; i < O::NOPS; ++i) {
     const unsigned op = O::op(i);
     if (!(op >> 31)) {
-      pl.get(int((op >> 4) & 255) - 128, int((op >> 12) & 15) - 8, w);
+      pl.get(int((op >> 4) & 255) - 128, int((op >> 12) & 4095) - 2048, w);
     } else if (op & 0x40000000u) {
       const int zi = (op >> 17) & 15;
       T* a = &acc[(U + NZ - zi) % NZ][(op >> 14) & 7][(op >> 12) & 3];
@@ -348,11 +361,33 @@ __device__ __forceinline__ void run_scatter(const L& pl, typename S::T (&acc)[S:
 
 // Store a thread tile (rows given by the merge mode) into global memory,
 // masked to the compute box; 128-bit stores when the whole vector is inside.
-template <class T, int VX, int M, bool CM, int BYS>
+// XS > 0: the M outputs are merged along x instead (2-D streaming views), XS
+// columns apart, all in row y0.
+template <class T, int VX, int M, bool CM, int BYS, int XS = 0>
 __device__ __forceinline__ void store_tile(T* __restrict__ out, const Grid& g, int z, int y0, int x0,
                                            const T (&acc)[M][VX]) {
-  const bool full_x = (x0 >= g.cx0) && (x0 + VX <= g.cx1) && g.vec_ok;
   T* const rp = mirror_plane<T>(g, z);
+  if constexpr (XS > 0) {
+    if (y0 < g.cy0 || y0 >= g.cy1) return;
+    T* row = out + z * g.sz + y0 * g.sy;
+#pragma unroll
+    for (int m = 0; m < M; ++m) {
+      const int xm = x0 + m * XS;
+      if (xm >= g.cx0 && xm + VX <= g.cx1 && g.vec_ok) {
+        stg_vec<T, VX>(row + xm, acc[m]);
+        if (rp) stg_vec<T, VX>(rp + y0 * g.sy + xm, acc[m]);
+      } else {
+#pragma unroll
+        for (int v = 0; v < VX; ++v)
+          if (xm + v >= g.cx0 && xm + v < g.cx1) {
+            row[xm + v] = acc[m][v];
+            if (rp) rp[y0 * g.sy + xm + v] = acc[m][v];
+          }
+      }
+    }
+    return;
+  }
+  const bool full_x = (x0 >= g.cx0) && (x0 + VX <= g.cx1) && g.vec_ok;
 #pragma unroll
   for (int m = 0; m < M; ++m) {
     const int y = CM ? y0 + m * BYS : y0 + m;
@@ -378,12 +413,12 @@ __device__ __forceinline__ void store_tile(T* __restrict__ out, const Grid& g, i
 // them from the Grid at run time) -- compile-time strides turn the per-plane
 // address arithmetic into immediates (no 64-bit multiplies, no constant-bank
 // reloads in the loop).
-template <class T, int VX, int M, bool CM, int BYS, i64 SY = 0, i64 SZ = 0>
+template <class T, int VX, int M, bool CM, int BYS, i64 SY = 0, i64 SZ = 0, int XS = 0>
 struct TileStore {
   T* base;             // element (plane 0, row y0, column x0)
   i64 sz_, rs_;        // plane stride, stride between the tile's rows (run-time strides)
-  unsigned rows;       // bit m: row m inside the compute box
-  bool full;           // whole vectors inside the compute box (128-bit stores)
+  unsigned rows;       // bit m: row m inside the compute box (XS > 0: output m's vector wholly inside)
+  bool full;           // whole vectors inside the compute box (XS > 0: row y0 inside)
   int x0, cx0, cx1;
   __device__ __forceinline__ i64 sz() const { return SZ ? SZ : sz_; }
   __device__ __forceinline__ i64 rs() const { return SY ? (CM ? BYS : 1) * SY : rs_; }
@@ -392,8 +427,15 @@ struct TileStore {
     base = out + (i64)y0 * (SY ? SY : g.sy) + x0;
     sz_ = g.sz;
     rs_ = (CM ? BYS : 1) * g.sy;
-    full = (x0 >= g.cx0) && (x0 + VX <= g.cx1) && g.vec_ok;
     rows = 0;
+    if constexpr (XS > 0) {      // merged along x (2-D streaming views)
+      full = y0 >= g.cy0 && y0 < g.cy1;
+#pragma unroll
+      for (int m = 0; m < M; ++m)
+        if (x0 + m * XS >= g.cx0 && x0 + m * XS + VX <= g.cx1 && g.vec_ok) rows |= 1u << m;
+      return;
+    }
+    full = (x0 >= g.cx0) && (x0 + VX <= g.cx1) && g.vec_ok;
 #pragma unroll
     for (int m = 0; m < M; ++m) {
       const int y = CM ? y0 + m * BYS : y0 + m;
@@ -407,6 +449,20 @@ struct TileStore {
     if (T* rp = mirror_plane<T>(g, z)) store_at(rp + (base - out), acc);
   }
   __device__ __forceinline__ void store_at(T* p, const T (&acc)[M][VX]) const {
+    if constexpr (XS > 0) {
+      if (!full) return;
+#pragma unroll
+      for (int m = 0; m < M; ++m) {
+        if (rows & (1u << m)) {
+          stg_vec<T, VX>(p + m * XS, acc[m]);
+        } else {
+#pragma unroll
+          for (int v = 0; v < VX; ++v)
+            if (x0 + m * XS + v >= cx0 && x0 + m * XS + v < cx1) p[m * XS + v] = acc[m][v];
+        }
+      }
+      return;
+    }
     if (full) {
 #pragma unroll
       for (int m = 0; m < M; ++m)
@@ -659,34 +715,49 @@ k_tiled(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, G
 //               prefetching: plane p+NS is requested while plane
 //               p+1.. are computed, hiding the per-iteration barrier.
 // ===========================================================================
+// Thread-tile geometry shared by the streaming families. y-merge (3-D): a
+// thread owns M rows (BM adjacent, CM BY apart) of VX columns. x-merge
+// (S::XM, 2-D streaming views whose planes are single rows): M vectors of one
+// row, adjacent (BM) or BX/M columns apart (CM).
+template <class S, int BX, int BY, int VX, int M, bool CM>
+struct TileGeom {
+  static constexpr int MY = S::XM ? 1 : M;                    // rows of the tile
+  static constexpr int TPX = S::XM ? BX / VX / M : BX / VX;   // threads along x
+  static constexpr int XS = S::XM ? (CM ? BX / M : VX) : 0;   // columns between merged outputs
+  static constexpr int XSTEP = S::XM && !CM ? VX * M : VX;   // columns between threads
+  static __device__ __forceinline__ int row(int ty) { return S::XM || CM ? ty : ty * M; }
+};
+
 template <class S, int BX, int BY, int VX, int M, bool CM, bool RT, int NS>
 struct StreamCfg {
   typedef typename S::T T;
+  typedef TileGeom<S, BX, BY, VX, M, CM> TG;
   static constexpr int ALN = (16 / (int)sizeof(T)) > VX ? (16 / (int)sizeof(T)) : VX;
   static constexpr int XOFF = ((S::XLO + ALN - 1) / ALN) * ALN;   // 16-byte aligned box start
   static constexpr int LX = ((XOFF + BX + S::XHI + ALN - 1) / ALN) * ALN;
-  static constexpr int LY = BY * M + S::YLO + S::YHI;
+  static constexpr int LY = BY * TG::MY + S::YLO + S::YHI;
   static constexpr int PLANE = ((LX * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
   static constexpr int NRING = (RT ? 1 : S::NZ) + NS - 1;
   static constexpr int SMEM = NRING * PLANE * (int)sizeof(T) + 8 * NRING + 128;
-  static constexpr int THREADS = (BX / VX) * BY;
+  static constexpr int THREADS = TG::TPX * BY;
 };
 
 template <class S, int BX, int BY, int VX, int M, bool CM, bool RT, int NS, bool TMA>
-__global__ void __launch_bounds__((BX / VX) * BY)
+__global__ void __launch_bounds__(StreamCfg<S, BX, BY, VX, M, CM, RT, NS>::THREADS)
 k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, Grid g, int chunk,
          const __grid_constant__ TmaDesc tmap) {
   typedef typename S::T T;
   typedef StreamCfg<S, BX, BY, VX, M, CM, RT, NS> C;
+  typedef typename C::TG TG;
   constexpr int NZ = S::NZ;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   T* ring = reinterpret_cast<T*>(smem_raw);
   unsigned long long* bar = reinterpret_cast<unsigned long long*>(smem_raw + C::NRING * C::PLANE * sizeof(T));
 
-  const int tid = threadIdx.y * (BX / VX) + threadIdx.x;
+  const int tid = threadIdx.y * TG::TPX + threadIdx.x;
   const int xa = (g.cx0 / C::ALN) * C::ALN;
   const int xb = xa + blockIdx.x * BX;
-  const int yb = g.cy0 + blockIdx.y * BY * M;
+  const int yb = g.cy0 + blockIdx.y * BY * TG::MY;
   const int zs = g.cz0 + blockIdx.z * chunk;
   const int ze = min(zs + chunk, g.cz1);
   const int pfirst = zs - S::ZLO;
@@ -739,11 +810,11 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
   }
 
   const int tx = threadIdx.x, ty = threadIdx.y;
-  const int row0 = S::YLO + (CM ? ty : ty * M);
-  const int col0 = C::XOFF + tx * VX;
-  const int x0 = xb + tx * VX;
-  const int y0 = yb + (CM ? ty : ty * M);
-  const TileStore<T, VX, M, CM, BY, S::SY, S::SZ> ts(out, g, y0, x0);
+  const int row0 = S::YLO + TG::row(ty);
+  const int col0 = C::XOFF + tx * TG::XSTEP;
+  const int x0 = xb + tx * TG::XSTEP;
+  const int y0 = yb + TG::row(ty);
+  const TileStore<T, VX, M, CM, BY, S::SY, S::SZ, TG::XS> ts(out, g, y0, x0);
 
   if constexpr (RT && S::RTSHIFT) {
     // large op tables (high-order stencils): one copy of the plane body and a
@@ -828,6 +899,7 @@ k_stream(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, 
 template <class S, int BX, int BY, int VX, int M, bool CM, bool RT, int NS, int TT>
 struct StreamTbCfg {
   typedef typename S::T T;
+  typedef TileGeom<S, BX, BY, VX, M, CM> TG;
   static constexpr int ALN = (16 / (int)sizeof(T)) > VX ? (16 / (int)sizeof(T)) : VX;
   // Column geometry. Without S::XSHIFT every ring uses the input plane's
   // geometry (column c = global xb - XOFF + c, XOFF rounded up to ALN). With
@@ -841,7 +913,7 @@ struct StreamTbCfg {
   static constexpr int XOFF = S::XSHIFT ? TT * S::XLO : ((TT * S::XLO + ALN - 1) / ALN) * ALN;
   static __device__ __forceinline__ constexpr int xoff(int s) { return S::XSHIFT ? (TT - s) * S::XLO : XOFF; }
   static constexpr int LX = ((XOFF + BX + TT * S::XHI + ALN - 1) / ALN) * ALN;
-  static constexpr int LY = BY * M + TT * (S::YLO + S::YHI);
+  static constexpr int LY = BY * TG::MY + TT * (S::YLO + S::YHI);
   static constexpr int PLANE = ((LX * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
   static constexpr int NIN = S::NZ + NS - 1;          // input ring (stage 0)
   static constexpr int NMID = S::NZ;                  // ring of each stage 1..TT-1
@@ -851,15 +923,16 @@ struct StreamTbCfg {
   static constexpr int PADF = 128 / (int)sizeof(T);
   static constexpr int PADB = ((MI * LX + ALN) * (int)sizeof(T) + 127) / 128 * 128 / (int)sizeof(T);
   static constexpr int SMEM = (PADF + (NIN + (TT - 1) * NMID) * PLANE + PADB) * (int)sizeof(T) + 8 * NIN + 128;
-  static constexpr int THREADS = (BX / VX) * BY;
+  static constexpr int THREADS = TG::TPX * BY;
 };
 
 template <class S, int BX, int BY, int VX, int M, bool CM, bool RT, int NS, int TT>
-__global__ void __launch_bounds__((BX / VX) * BY)
+__global__ void __launch_bounds__(StreamTbCfg<S, BX, BY, VX, M, CM, RT, NS, TT>::THREADS)
 k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, Grid g, int chunk,
             const __grid_constant__ TmaDesc tmap) {
   typedef typename S::T T;
   typedef StreamTbCfg<S, BX, BY, VX, M, CM, RT, NS, TT> C;
+  typedef typename C::TG TG;
   constexpr int NZ = S::NZ;
   constexpr int MI = C::MI;
   static_assert(TT >= 2, "k_stream_tb needs TT >= 2");
@@ -869,10 +942,10 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
   unsigned long long* bar = reinterpret_cast<unsigned long long*>(
       smem_raw + (C::PADF + (C::NIN + (TT - 1) * C::NMID) * C::PLANE + C::PADB) * sizeof(T));
 
-  const int tid = threadIdx.y * (BX / VX) + threadIdx.x;
+  const int tid = threadIdx.y * TG::TPX + threadIdx.x;
   const int xa = (g.cx0 / C::ALN) * C::ALN;
   const int xb = xa + blockIdx.x * BX;
-  const int yb = g.cy0 + blockIdx.y * BY * M;
+  const int yb = g.cy0 + blockIdx.y * BY * TG::MY;
   const int zs = g.cz0 + blockIdx.z * chunk;
   const int ze = min(zs + chunk, g.cz1);
   const int pin0 = zs - TT * S::ZLO;                   // first input plane
@@ -918,7 +991,7 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
     constexpr int HY0 = (TT - s) * S::YLO, HY1 = (TT - s) * S::YHI;
     constexpr int TXL = ((HX0 + VX - 1) / VX) * VX;
     constexpr int NTX = (TXL + BX + HX1 + VX - 1) / VX;
-    constexpr int RY = BY * M + HY0 + HY1;
+    constexpr int RY = BY * TG::MY + HY0 + HY1;
     constexpr int NTY = (RY + MI - 1) / MI;
     if (it < s * (NZ - 1)) return;
     const int q = pin0 + it - s * S::ZHI;
@@ -929,7 +1002,7 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
 #pragma unroll
     for (int zi = 0; zi < NZ; ++zi) src[zi] = stage_plane(s - 1, q + zi - S::ZLO);
     const bool zupd = q >= g.uz0 && q < g.uz1;
-    const int rx0 = xb - HX0, rx1 = xb + BX + HX1, ry0 = yb - HY0, ry1 = yb + BY * M + HY1;
+    const int rx0 = xb - HX0, rx1 = xb + BX + HX1, ry0 = yb - HY0, ry1 = yb + BY * TG::MY + HY1;
     for (int t = tid; t < NTX * NTY; t += C::THREADS) {
       const int gx0 = xb - TXL + (t % NTX) * VX, gy0 = ry0 + (t / NTX) * MI;
       const int lbase = (gy0 - Y0) * C::LX + (gx0 - X0);
@@ -961,10 +1034,10 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
   };
 
   const int tx = threadIdx.x, ty = threadIdx.y;
-  const int row0 = TT * S::YLO + (CM ? ty : ty * M);
-  const int col0 = C::XOFF + tx * VX;
-  const int x0 = xb + tx * VX;
-  const int y0 = yb + (CM ? ty : ty * M);
+  const int row0 = TT * S::YLO + TG::row(ty);
+  const int col0 = C::XOFF + tx * TG::XSTEP;
+  const int x0 = xb + tx * TG::XSTEP;
+  const int y0 = yb + TG::row(ty);
 
   // one pipeline iteration up to (excluding) the last stage
   auto front = [&](int it) {
@@ -1002,7 +1075,7 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
         if constexpr (S::RTSHIFT) {                      // one body + register shift (see k_stream)
           (void)ur;
           run_scatter<S, VX, M, NZ - 1>(pl, acc);
-          if (z >= zs) store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc[0]);
+          if (z >= zs) store_tile<T, VX, M, CM, BY, TG::XS>(out, g, z, y0, x0, acc[0]);
           shift_queue<T, NZ, M, VX>(acc);
         } else {
           static_for<0, NZ>([&](auto ic) {
@@ -1010,7 +1083,7 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
             if (ur == UR) {
               zero_acc<T, VX, M>(acc[UR]);
               run_scatter<S, VX, M, UR>(pl, acc);
-              if (z >= zs) store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc[(UR + 1) % NZ]);
+              if (z >= zs) store_tile<T, VX, M, CM, BY, TG::XS>(out, g, z, y0, x0, acc[(UR + 1) % NZ]);
             }
           });
         }
@@ -1029,7 +1102,7 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
 #pragma unroll
         for (int zi = 0; zi < NZ; ++zi) pl[zi].p = stage_plane(TT - 1, z + zi - S::ZLO) + row0 * C::LX + col0;
         run_gather<S, VX, M>(pl, acc);
-        store_tile<T, VX, M, CM, BY>(out, g, z, y0, x0, acc);
+        store_tile<T, VX, M, CM, BY, TG::XS>(out, g, z, y0, x0, acc);
       }
       __syncthreads();
     }
@@ -1075,6 +1148,7 @@ k_stream_tb(const typename S::T* __restrict__ in, typename S::T* __restrict__ ou
 // ===========================================================================
 template <class S, int BX, int BY, int VX, int M, int TT, int MI, int s>
 struct TbRtStage {
+  static constexpr int MY = S::XM ? 1 : M;                 // rows of the output tile
   static constexpr int HX0 = (TT - s) * S::XLO, HX1 = (TT - s) * S::XHI;
   static constexpr int HY0 = (TT - s) * S::YLO, HY1 = (TT - s) * S::YHI;
   // tile x origin = xb - TXL (S::XSHIFT: exactly the region's left edge, see StreamTbRtCfg)
@@ -1084,7 +1158,7 @@ struct TbRtStage {
   static constexpr int VXM = S::MVX;
   static constexpr int TXL = S::XSHIFT ? HX0 : ((HX0 + VXM - 1) / VXM) * VXM;
   static constexpr int NTX = (TXL + BX + HX1 + VXM - 1) / VXM;
-  static constexpr int RY = BY * M + HY0 + HY1;
+  static constexpr int RY = BY * MY + HY0 + HY1;
   static constexpr int NTY = (RY + MI - 1) / MI;
   static constexpr int NT = NTX * NTY;
   static constexpr int W = (NT + 31) / 32;                 // warps of group s
@@ -1102,6 +1176,7 @@ struct TbRtWarp0<S, BX, BY, VX, M, TT, MI, 1> { static constexpr int value = 1; 
 template <class S, int BX, int BY, int VX, int M, bool CM, int NS, int TT>
 struct StreamTbRtCfg {
   typedef typename S::T T;
+  typedef TileGeom<S, BX, BY, VX, M, CM> TG;
   static constexpr int ALN = (16 / (int)sizeof(T)) > VX ? (16 / (int)sizeof(T)) : VX;
   // Column geometry. Without S::XSHIFT every ring uses the input plane's
   // geometry (column c = global xb - XOFF + c, XOFF rounded up to ALN). With
@@ -1115,7 +1190,7 @@ struct StreamTbRtCfg {
   static constexpr int XOFF = S::XSHIFT ? TT * S::XLO : ((TT * S::XLO + ALN - 1) / ALN) * ALN;
   static __device__ __forceinline__ constexpr int xoff(int s) { return S::XSHIFT ? (TT - s) * S::XLO : XOFF; }
   static constexpr int LX = ((XOFF + BX + TT * S::XHI + ALN - 1) / ALN) * ALN;
-  static constexpr int LY = BY * M + TT * (S::YLO + S::YHI);
+  static constexpr int LY = BY * TG::MY + TT * (S::YLO + S::YHI);
   static constexpr int PLANE = ((LX * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
   static constexpr int MI = S::MI;
   static constexpr int PADF = 128 / (int)sizeof(T);
@@ -1125,7 +1200,7 @@ struct StreamTbRtCfg {
   static constexpr int ELEMS = PADF + (NR + MR * (TT - 1)) * PLANE + PADB;
   static constexpr int NBAR = 2 * NR + 2 * MR * (TT - 1);
   static constexpr int SMEM = ELEMS * (int)sizeof(T) + 8 * NBAR + 128;
-  static constexpr int FT = (BX / VX) * BY;                 // last-stage tiles
+  static constexpr int FT = TG::TPX * BY;                   // last-stage tiles
   static constexpr int WF = (FT + 31) / 32;
   // register split (S::REG_LO > 0): producer + intermediate stages give
   // registers to the last stage (setmaxnreg); role boundaries are then
@@ -1160,9 +1235,10 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
 
   const int tid = threadIdx.x;
   const int warp = tid >> 5;
+  constexpr int AL = S::ELECT ? 1 : 32;                // arrivals per consumer warp
   const int xa = (g.cx0 / C::ALN) * C::ALN;
   const int xb = xa + blockIdx.x * BX;
-  const int yb = g.cy0 + blockIdx.y * BY * M;
+  const int yb = g.cy0 + blockIdx.y * BY * C::TG::MY;
   const int zs = g.cz0 + blockIdx.z * chunk;
   const int ze = min(zs + chunk, g.cz1);
   const int pin0 = zs - TT * S::ZLO;                   // first input plane
@@ -1175,14 +1251,14 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     if constexpr (S::TMA) tma_prefetch_desc(&tmap);
     for (int q = 0; q < NR; ++q) {
       mbar_init(&full_in[q], S::TMA ? 1 : 32);   // cp.async: one arrival per producer lane
-      mbar_init(&empty_in[q], 32 * TbRtStage<S, BX, BY, VX, M, TT, MI, 1>::W);
+      mbar_init(&empty_in[q], AL * TbRtStage<S, BX, BY, VX, M, TT, MI, 1>::W);
     }
     static_for<1, TT>([&](auto sc) {
       constexpr int s = decltype(sc)::value;
       constexpr int WN = s + 1 < TT ? TbRtStage<S, BX, BY, VX, M, TT, MI, s + 1>::W : C::WF;
       for (int b = 0; b < MR; ++b) {
-        mbar_init(&full_s(s)[b], 32 * TbRtStage<S, BX, BY, VX, M, TT, MI, s>::W);
-        mbar_init(&empty_s(s)[b], 32 * WN);
+        mbar_init(&full_s(s)[b], AL * TbRtStage<S, BX, BY, VX, M, TT, MI, s>::W);
+        mbar_init(&empty_s(s)[b], AL * WN);
       }
     });
     fence_mbar_init();
@@ -1231,12 +1307,20 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     constexpr bool XOVER = XO_W - G::TXL + G::NTX * MV > C::LX;
     const int t = tid - 32 * W0;
     const bool act = t < G::NT;
-    const int gx0 = xb - G::TXL + (t % G::NTX) * MV;
-    const int gy0 = yb - G::HY0 + (t / G::NTX) * MI;
+    // tile (column cx, row cy) of thread t. S::WALIGN: the first NXM columns of
+    // every tile row (a multiple of 32) are whole warps of one tile row, the
+    // remaining NTX - NXM columns of all rows go to the last warp(s); otherwise
+    // row-major over NTX columns, where a warp straddling two tile rows hits
+    // the same banks twice (a third shared-memory wavefront per access)
+    constexpr int NXM = S::WALIGN ? (G::NTX / 32) * 32 : 0, NXE = G::NTX - NXM;
+    const int cx = t < NXM * G::NTY ? t % (NXM ? NXM : 1) : NXM + (t - NXM * G::NTY) % NXE;
+    const int cy = t < NXM * G::NTY ? t / (NXM ? NXM : 1) : (t - NXM * G::NTY) / NXE;
+    const int gx0 = xb - G::TXL + cx * MV;
+    const int gy0 = yb - G::HY0 + cy * MI;
     const int lb_r = (gy0 - Y0) * C::LX + (gx0 - xb + XO_R);   // tile origin in the source ring
     const int lrow = gy0 - Y0, lcol = gx0 - xb + XO_W;
     const int lb = lrow * C::LX + lcol;                         // ... in the stage's own ring
-    const int ry1 = yb + BY * M + G::HY1;
+    const int ry1 = yb + BY * G::MY + G::HY1;
     // rows: bit m = writable (inside R_s rows and the array), bit 8+m = inside the update box
     unsigned rows = 0, allup = 1;
 #pragma unroll
@@ -1272,7 +1356,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
           SmemPlane<T, MV, C::LX> pl{src + lb_r - S::XSH};
           run_scatter_ops<S, typename S::Mid, MV, MI, U>(pl, acc);
         }
-        if (s > 1) mbar_arrive(&ein[si]);                // input slot read (stage 1: below)
+        if (s > 1) warp_arrive<S::ELECT>(&ein[si]);      // input slot read (stage 1: below)
         const int so = j % MR;
         T* dst = mid + (MR * (s - 1) + so) * C::PLANE;
         if (j >= MR) mbar_wait_sleep(&empty_s(s)[so], (unsigned)((j / MR - 1) & 1));
@@ -1316,8 +1400,8 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
             }
           }
         }
-        if (s == 1 && j >= S::ZHI) mbar_arrive(&ein[(j - S::ZHI) % NR]);   // frame source released
-        mbar_arrive(&full_s(s)[so]);                     // stage-s plane written
+        if (s == 1 && j >= S::ZHI) warp_arrive<S::ELECT>(&ein[(j - S::ZHI) % NR]);   // frame source released
+        warp_arrive<S::ELECT>(&full_s(s)[so]);           // stage-s plane written
         if constexpr (S::RTSHIFT) shift_queue<T, NZ, MI, MV>(acc);
       });
     }
@@ -1328,12 +1412,13 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
   {
     const int q = tid - 32 * C::WL;
     const bool act = q < C::FT;
-    const int tx = q % (BX / VX), ty = q / (BX / VX);
-    const int row0 = TT * S::YLO + (CM ? ty : ty * M);
-    const int col0 = C::xoff(TT - 1) + tx * VX - S::XSH;   // window start in the last ring
-    const int x0 = xb + tx * VX;
-    const int y0 = yb + (CM ? ty : ty * M);
-    const TileStore<T, VX, M, CM, BY, S::SY, S::SZ> ts(out, g, y0, x0);
+    typedef typename C::TG TG;
+    const int tx = q % TG::TPX, ty = q / TG::TPX;
+    const int row0 = TT * S::YLO + TG::row(ty);
+    const int col0 = C::xoff(TT - 1) + tx * TG::XSTEP - S::XSH;   // window start in the last ring
+    const int x0 = xb + tx * TG::XSTEP;
+    const int y0 = yb + TG::row(ty);
+    const TileStore<T, VX, M, CM, BY, S::SY, S::SZ, TG::XS> ts(out, g, y0, x0);
     unsigned long long* fin = full_s(TT - 1);
     unsigned long long* ein = empty_s(TT - 1);
     T acc[NZ][M][VX];
@@ -1359,7 +1444,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
             run_scatter<S, VX, M, U>(pl, acc);
           }
         }
-        mbar_arrive(&ein[si]);
+        warp_arrive<S::ELECT>(&ein[si]);
         const int z = pin0 + j - TT * S::ZHI;
         if (act && z >= zs) ts.store(z, acc[(U + 1) % NZ], g, out);
         if constexpr (S::RTSHIFT) shift_queue<T, NZ, M, VX>(acc);

@@ -145,6 +145,14 @@ static void default_params(uint32_t oc, int ndim, int dtype, stencil_params_t* p
   } else {
     p->vx = vmax; p->bx = 32 * vmax; p->by = merge ? 4 : 8; p->bz = 1;
   }
+  if (ndim == 2 && (fam == FAM_STREAM || fam == FAM_STREAM_TB) && merge) {
+    // 2-D streaming views merge along x (resolve_variant): 2 vectors of <= 16
+    // bytes per thread and 32 threads per tile row -> 128-column tiles, whose
+    // TMA box (with the halo) stays within 256 elements
+    p->merge = 2;
+    p->vx = std::min(vmax, 2);
+    p->bx = 32 * p->vx * p->merge;
+  }
 }
 
 // counter-based hash for the seeded settings sampler
@@ -245,12 +253,12 @@ static TmaBox tma_box(const Variant& v, const Pattern& p, int elem) {
   auto ru = [](int a, int b) { return (a + b - 1) / b * b; };
   if (v.family == FAM_TILED) {
     const int xoff = ru(v.tt * p.xlo, aln);
-    return {ru(xoff + v.bx + v.tt * p.xhi, aln), v.by * v.m + v.tt * (p.ylo + p.yhi),
+    return {ru(xoff + v.bx + v.tt * p.xhi, aln), v.rows() + v.tt * (p.ylo + p.yhi),
             v.bz + v.tt * (p.zlo + p.zhi)};
   }
   const int t = v.family == FAM_STREAM_TB ? v.tt : 1;   // stream: halo of t time steps
   const int xoff = v.xshift ? t * p.xlo : ru(t * p.xlo, aln);   // mirrors StreamTbRtCfg::XOFF
-  return {ru(xoff + v.bx + t * p.xhi, aln), v.by * v.m + t * (p.ylo + p.yhi), 1};
+  return {ru(xoff + v.bx + t * p.xhi, aln), v.rows() + t * (p.ylo + p.yhi), 1};
 }
 
 // Register split of the warp-specialised ST_TB_RT kernel (setmaxnreg): the
@@ -298,7 +306,10 @@ static int resolve_variant(stencil_plan_s* P) {
   if (fam == FAM_NAIVE) { v.vx = 1; v.bz = 1; }
   if (fam == FAM_STREAM || fam == FAM_STREAM_TB) v.bz = 1;
   if (P->ndim == 2) {
-    if (fam == FAM_STREAM || fam == FAM_STREAM_TB) { v.by = 1; v.m = 1; }
+    // 2-D streaming views [ny][1][nx]: a plane is one row, so BM / CM merge
+    // along x, the only other axis (P:L63 names merging in the
+    // innermost dimension as a real, coalescing-relevant choice)
+    if (fam == FAM_STREAM || fam == FAM_STREAM_TB) { v.by = 1; v.flat = true; v.xm = v.m > 1; }
     else v.bz = 1;
   }
   if (v.vx != 1 && v.vx != 2 && v.vx != 4) SM_FAIL(STENCIL_E_INVAL, "vx must be 1, 2 or 4");
@@ -307,6 +318,9 @@ static int resolve_variant(stencil_plan_s* P) {
     SM_FAIL(STENCIL_E_INVAL, "tile parameters must be powers of two (bx=%d by=%d bz=%d merge=%d vx=%d)", v.bx,
             v.by, v.bz, v.m, v.vx);
   if (v.m > 8) SM_FAIL(STENCIL_E_INVAL, "merge factor must be <= 8");
+  if (v.xm && v.bx < v.vx * v.m)
+    SM_FAIL(STENCIL_E_OC_INFEASIBLE, "x-merge of %d vectors of %d needs a tile of >= %d columns (bx=%d)", v.m, v.vx,
+            v.vx * v.m, v.bx);
   if (v.tt < 1 || v.tt > 8) SM_FAIL(STENCIL_E_INVAL, "tb_steps must be in 1..8");
   if (v.ns < 1 || v.ns > 8) SM_FAIL(STENCIL_E_INVAL, "pr_stages must be in 1..8");
   if (fam == FAM_STREAM_TB && v.rt && v.tt >= 2) {
@@ -536,8 +550,8 @@ static int launch_sweep(stencil_plan_s* P, const Variant& v, const Kernel& k, co
   } else {
     const int xa = (g.cx0 / aln) * aln;
     gx = (g.cx1 - xa + v.bx - 1) / v.bx;
-    gy = (cylen + v.by * v.m - 1) / (v.by * v.m);
-    bx = v.bx / v.vx; by = v.by;
+    gy = (cylen + v.rows() - 1) / v.rows();
+    bx = v.family == FAM_TILED ? v.bx / v.vx : v.tpx(); by = v.by;
     if (v.family == FAM_STREAM_TB && v.rt) { bx = v.threads(); by = 1; }   // warp-specialised, 1-D
     if (v.tma) SM_TRY(get_tmap(P, v, src, &tm));
     if (v.family == FAM_TILED) {

@@ -125,7 +125,7 @@ int Variant::threads() const {
   if (family == FAM_STREAM_TB && rt) return ws_threads;
   switch (family) {
     case FAM_NAIVE: return bx * by;
-    default: return (bx / vx) * by;
+    default: return (family == FAM_TILED ? bx / vx : tpx()) * by;
   }
 }
 
@@ -136,6 +136,7 @@ static int roundup(int a, int b) { return (a + b - 1) / b * b; }
 // retiming pipeline need ~95 registers and lose 15% to the lower occupancy.
 int Variant::mid_rows(const Pattern& p, int elem) const {
   (void)p; (void)elem;
+  if (flat) return 1;          // 2-D streaming view: a plane is one row, taller tiles only waste lanes
   if (family == FAM_STREAM_TB && rt)
     if (const char* e = getenv("STENCIL_MID_ROWS")) return atoi(e);   // dev override
   return midvx == 1 ? 4 : 2;   // scalar-column intermediate tiles: 1 x 4
@@ -177,12 +178,12 @@ int Variant::tbrt_threads(const Pattern& p, int elem, int* wl_out) const {
     const int mvx = midvx > 0 ? midvx : vx;
     const int txl = xshift ? hx0 : roundup(hx0, mvx);
     const int ntx = (txl + bx + hx1 + mvx - 1) / mvx;
-    const int nty = (by * m + hy0 + hy1 + mi - 1) / mi;
+    const int nty = (rows() + hy0 + hy1 + mi - 1) / mi;
     warps += (ntx * nty + 31) / 32;
   }
   if (reg_lo > 0) warps = roundup(warps, 4);    // warpgroup-aligned roles (register split)
   *wl_out = warps;
-  warps += ((bx / vx) * by + 31) / 32;
+  warps += (tpx() * by + 31) / 32;
   if (reg_lo > 0) warps = roundup(warps, 4);
   return 32 * warps;
 }
@@ -202,7 +203,7 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
   if (family == FAM_STREAM) {
     const int xoff = roundup(p.xlo, aln);
     const int lx = roundup(xoff + bx + p.xhi, aln);
-    const int ly = by * m + p.ylo + p.yhi;
+    const int ly = rows() + p.ylo + p.yhi;
     const int plane = roundup(lx * ly * elem, 128) / elem;
     const int nz = p.zlo + p.zhi + 1;
     const int nring = (rt ? 1 : nz) + ns - 1;
@@ -211,7 +212,7 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
   if (family == FAM_STREAM_TB && rt) {   // mirrors StreamTbRtCfg
     const int xoff = xshift ? tt * p.xlo : roundup(tt * p.xlo, aln);
     const int lx = roundup(xoff + bx + tt * p.xhi, aln);
-    const int ly = by * m + tt * (p.ylo + p.yhi);
+    const int ly = rows() + tt * (p.ylo + p.yhi);
     const int plane = roundup(lx * ly * elem, 128) / elem;
     const int padf = 128 / elem;
     const int padb = roundup((mid_rows(p, elem) * lx + aln) * elem, 128) / elem;
@@ -221,7 +222,7 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
   if (family == FAM_STREAM_TB) {   // mirrors StreamTbCfg
     const int xoff = roundup(tt * p.xlo, aln);
     const int lx = roundup(xoff + bx + tt * p.xhi, aln);
-    const int ly = by * m + tt * (p.ylo + p.yhi);
+    const int ly = rows() + tt * (p.ylo + p.yhi);
     const int plane = roundup(lx * ly * elem, 128) / elem;
     const int nz = p.zlo + p.zhi + 1;
     const int nin = nz + ns - 1;
@@ -253,31 +254,37 @@ static std::vector<uint32_t> encode_ops(const Pattern& pat, const Variant& v, bo
   const int VX = v.family == FAM_NAIVE ? 1 : v.vx;
   const int M = v.m, BY = v.by;
   const bool scatter = v.rt && (v.family == FAM_STREAM || v.family == FAM_STREAM_TB);
+  // placement of merged output m relative to the thread's first output: rows
+  // (y-merge: BM m, CM m*BY) or vectors (x-merge: BM m, CM m*BX/M/VX)
+  const int KS = v.xm ? (v.cm ? v.bx / M / VX : 1) : 0;
+  auto rsh = [&](int m) { return v.xm ? 0 : (v.cm ? m * BY : m); };
+  auto csh = [&](int m) { return v.xm ? m * KS : 0; };
   // window vector kv covers columns [kv*VX - xsh, kv*VX - xsh + VX) relative to
   // the thread's first output column (xsh > 0: TB-RT aligned windows, StreamTbRtCfg)
   const int xsh = v.xshift ? pat.xlo % VX : 0;
   auto fdiv = [](int a, int b) { return a >= 0 ? a / b : -((-a + b - 1) / b); };
   const int KLO = fdiv(xsh - pat.xlo, VX), KHI = fdiv(VX - 1 + pat.xhi + xsh, VX);
   auto load = [](int zi, int j, int kv) {
-    return (uint32_t)(zi & 15) | ((uint32_t)(j + 128) & 255) << 4 | ((uint32_t)(kv + 8) & 15) << 12;
+    return (uint32_t)(zi & 15) | ((uint32_t)(j + 128) & 255) << 4 | ((uint32_t)(kv + 2048) & 4095) << 12;
   };
   auto fma = [](int id, int e, int vv, int m, int zi) {
     return 0x80000000u | (uint32_t)id | (uint32_t)e << 10 | (uint32_t)vv << 12 | (uint32_t)m << 14 |
            (uint32_t)zi << 17;
   };
   std::vector<uint32_t> ops, f;
-  auto window = [&](int zsel, int j_rel, int kv, int zi_lo, int zi_hi, int m_lo, int m_hi, int jbase) {
-    // FMAs fed by window (row j_rel, vector kv); jbase = j_rel - (row of output m_lo's dy = 0)
+  auto window = [&](int zsel, int j_rel, int kv, int zi_lo, int zi_hi, int m_lo, int m_hi) {
+    // FMAs fed by window (row j_rel, vector kv) into outputs m_lo..m_hi-1
     f.clear();
     for (int zi = zi_lo; zi < zi_hi; ++zi)
       for (int m = m_lo; m < m_hi; ++m) {
-        const int dyi = (v.cm ? jbase : jbase - m) + pat.ylo;
-        // element e of this window feeds column vv through offset dx = kv*VX + e - vv
+        const int dyi = j_rel - rsh(m) + pat.ylo;
+        // element e of this window feeds column vv of output m through offset
+        // dx = (kv - csh(m))*VX + e - vv - xsh
         for (int d = kv * VX - xsh - (VX - 1); d <= kv * VX - xsh + VX - 1; ++d)
           for (int vv = 0; vv < VX; ++vv) {
             const int e = d - kv * VX + xsh + vv;
             if (e < 0 || e >= VX) continue;
-            const int id = cidx(zi, dyi, d + pat.xlo);
+            const int id = cidx(zi, dyi, d - csh(m) * VX + pat.xlo);
             if (id < 0) continue;
             if (pair && !(vv & 1) && !(e & 1) && vv + 1 < VX && e + 1 < VX) {
               f.push_back(fma(id, e, vv, m, zi) | 0x40000000u);   // columns vv, vv+1
@@ -292,25 +299,38 @@ static std::vector<uint32_t> encode_ops(const Pattern& pat, const Variant& v, bo
       ops.insert(ops.end(), f.begin(), f.end());
     }
   };
-  if (!v.cm) {
+  // (windows are visited in (zi, row, vector) order, and each window emits its
+  // FMAs in ascending dx: every accumulator's chain is lexicographic)
+  if (v.xm && !v.cm) {           // x-BM: outputs share windows over M + extent vectors
+    for (int zi = 0; zi < (scatter ? 1 : NZ); ++zi)
+      for (int j = -pat.ylo; j <= pat.yhi; ++j)
+        for (int kv = KLO; kv <= KHI + M - 1; ++kv)
+          window(zi, j, kv, scatter ? 0 : zi, scatter ? NZ : zi + 1, 0, M);
+  } else if (v.xm) {             // x-CM: separate windows per output, KS vectors apart
+    for (int zi = 0; zi < (scatter ? 1 : NZ); ++zi)
+      for (int m = 0; m < M; ++m)
+        for (int j = -pat.ylo; j <= pat.yhi; ++j)
+          for (int kv = KLO; kv <= KHI; ++kv)
+            window(zi, j, kv + m * KS, scatter ? 0 : zi, scatter ? NZ : zi + 1, m, m + 1);
+  } else if (!v.cm) {
     if (!scatter) {
       for (int zi = 0; zi < NZ; ++zi)
         for (int j = -pat.ylo; j < M + pat.yhi; ++j)
-          for (int kv = KLO; kv <= KHI; ++kv) window(zi, j, kv, zi, zi + 1, 0, M, j);
+          for (int kv = KLO; kv <= KHI; ++kv) window(zi, j, kv, zi, zi + 1, 0, M);
     } else {
       for (int j = -pat.ylo; j < M + pat.yhi; ++j)
-        for (int kv = KLO; kv <= KHI; ++kv) window(0, j, kv, 0, NZ, 0, M, j);
+        for (int kv = KLO; kv <= KHI; ++kv) window(0, j, kv, 0, NZ, 0, M);
     }
   } else {
     if (!scatter) {
       for (int zi = 0; zi < NZ; ++zi)
         for (int m = 0; m < M; ++m)
           for (int j = -pat.ylo; j <= pat.yhi; ++j)
-            for (int kv = KLO; kv <= KHI; ++kv) window(zi, m * BY + j, kv, zi, zi + 1, m, m + 1, j);
+            for (int kv = KLO; kv <= KHI; ++kv) window(zi, m * BY + j, kv, zi, zi + 1, m, m + 1);
     } else {
       for (int m = 0; m < M; ++m)
         for (int j = -pat.ylo; j <= pat.yhi; ++j)
-          for (int kv = KLO; kv <= KHI; ++kv) window(0, m * BY + j, kv, 0, NZ, m, m + 1, j);
+          for (int kv = KLO; kv <= KHI; ++kv) window(0, m * BY + j, kv, 0, NZ, m, m + 1);
     }
   }
   return ops;
@@ -322,7 +342,7 @@ int count_window_loads(const Pattern& pat, int elem, const Variant& v) {
   int n = 0;
   for (uint32_t op : encode_ops(pat, v, false)) n += !(op >> 31);
   Variant vm = v;
-  vm.family = FAM_STREAM; vm.cm = false; vm.m = v.mid_rows(pat, elem);
+  vm.family = FAM_STREAM; vm.cm = false; vm.xm = false; vm.m = v.mid_rows(pat, elem);
   if (v.midvx > 0) vm.vx = v.midvx;
   for (uint32_t op : encode_ops(pat, vm, false)) n += !(op >> 31);
   return n;
@@ -375,12 +395,12 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   const int tmid = v.family == FAM_TILED && v.tt > 1 ? v.tiled_mid : 0;
   if (tmid > 0) {                      // k_tiled intermediate steps: 1 x tmid tiles, gather
     Variant vm = v;
-    vm.family = FAM_STREAM; vm.rt = false; vm.cm = false; vm.m = tmid; vm.vx = 1; vm.xshift = false;
+    vm.family = FAM_STREAM; vm.rt = false; vm.cm = false; vm.xm = false; vm.m = tmid; vm.vx = 1; vm.xshift = false;
     mops = encode_ops(pat, vm, pair);
   }
   if (v.family == FAM_STREAM_TB) {     // intermediate fused steps: VX x MI tiles, gather or (RT) scatter
     Variant vm = v;
-    vm.family = FAM_STREAM; vm.cm = false; vm.m = mi;
+    vm.family = FAM_STREAM; vm.cm = false; vm.xm = false; vm.m = mi;
     if (v.midvx > 0) vm.vx = v.midvx;
     mops = encode_ops(pat, vm, pair);
   }
@@ -397,6 +417,13 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   o << "  static constexpr int TMID = " << tmid << ";\n";
   o << "  static constexpr int MVX = " << (v.midvx > 0 ? v.midvx : std::max(v.vx, 1)) << ";\n";
   o << "  static constexpr bool SPLITMID = " << (v.splitmid ? "true" : "false") << ";\n";
+  {   // k_stream_tb_rt hand-off details (dev overrides for A/B measurements)
+    const char* el = getenv("STENCIL_ELECT");
+    const char* wa = getenv("STENCIL_WALIGN");
+    o << "  static constexpr bool ELECT = " << ((el ? atoi(el) : 1) ? "true" : "false") << ";\n";
+    o << "  static constexpr bool WALIGN = " << ((wa ? atoi(wa) : 1) ? "true" : "false") << ";\n";
+  }
+  o << "  static constexpr bool XM = " << (v.xm ? "true" : "false") << ";   // merge along x (2-D streaming)\n";
   o << "  static constexpr bool TMA = " << (v.tma ? "true" : "false") << ";   // streaming TB staging (else cp.async)\n";
   o << "  static constexpr bool XSHIFT = " << (v.xshift ? "true" : "false") << ";\n";
   o << "  static constexpr int XSH = " << (v.xshift ? pat.xlo % std::max(v.vx, 1) : 0) << ";\n";

@@ -89,7 +89,11 @@ struct Variant {
   bool splitmid = false;      // k_stream_tb_rt: even/odd-split rows in the last intermediate ring
   int midvx = 0;              // k_stream_tb_rt: columns per thread of the intermediate steps (0 = vx)
   int tiled_mid = 0;          // k_tiled (TB): rows of the 1 x n intermediate-step register tiles (0 = scalar)
+  bool flat = false;          // 2-D streaming view [ny][1][nx]: every plane is one row
+  bool xm = false;            // merging (BM/CM, factor m) along x instead of y (2-D streaming view)
   std::string name_expr(const char* desc) const;
+  int rows() const { return xm ? by : by * m; }          // output rows of a CTA tile
+  int tpx() const { return xm ? bx / vx / m : bx / vx; }  // threads along x (streaming families)
   int threads() const;
   int smem_bytes(const Pattern& p, int elem) const;
   int mid_rows(const Pattern& p, int elem) const;

@@ -195,3 +195,21 @@ def test_tbrt_aligned_window_choice():
     assert not _plan((64, 64, 64), acc, c, "f64", oc, prm).info["xshift"]
     assert not _plan((64, 64, 64), acc, c, "f32", oc).info["xshift"]
     assert not _plan((64, 64, 64), acc, c, "f64", sm.oc_from_name("ST_BM_RT_PR")).info["xshift"]
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_2d_streaming_merge_along_x(dtype):
+    """2-D streaming views (planes are single rows) merge BM / CM along x
+    (P:L55-L56): ST, ST_BM and ST_CM (and their RT/PR/TB siblings) are
+    distinct kernels, each covering the same tile with fewer, wider threads."""
+    acc, c = si.config_stencil("random2d:2:4")
+    dims = (300, 520)
+    for suffix in ("", "_RT_PR", "_TB_RT"):
+        plans = {m: sm.Plan(dims, acc, c, dtype, sm.oc_from_name("ST" + m + suffix))
+                 for m in ("", "_BM", "_CM")}
+        names = {m: p.info["kernel_name"] for m, p in plans.items()}
+        assert len(set(names.values())) == 3, names
+        base, bm = plans[""].info, plans["_BM"].info
+        assert bm["params"]["merge"] == 2 and base["params"]["merge"] == 1
+        if suffix != "_TB_RT":
+            assert bm["threads"] * bm["params"]["vx"] * 2 == bm["params"]["bx"]
