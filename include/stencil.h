@@ -86,7 +86,9 @@ typedef struct {
     int32_t by;           /* threads per CTA along y (power of two) */
     int32_t bz;           /* non-streaming tiled kernels: output planes per CTA */
     int32_t vx;           /* outputs per thread along x (1, 2, 4): one 128-bit vector */
-    int32_t merge;        /* BM/CM merge factor k (outputs per thread along y; 1..8) */
+    int32_t merge;        /* BM/CM merge factor k (1..8): outputs per thread along y; in 2-D
+                             streaming OCs (planes are single rows) along x -- BM adjacent
+                             vectors, CM vectors bx/k columns apart */
     int32_t stream_chunk; /* ST: output planes per CTA ("concurrent streaming") */
     int32_t tb_steps;     /* TB: time steps fused per launch (2..8) */
     int32_t pr_stages;    /* PR: planes in flight in the TMA pipeline (1..8; the settings
@@ -104,7 +106,9 @@ typedef struct {
     int32_t smem_bytes;       /* dynamic shared memory per CTA */
     int32_t threads;          /* threads per CTA */
     int32_t regs;             /* registers per thread of the main kernel (0 until compiled) */
-    int32_t uses_tma;         /* 1 if halo tiles are staged with cp.async.bulk.tensor */
+    int32_t uses_tma;         /* 1 if halo tiles are staged with cp.async.bulk.tensor; 0 =
+                                 element-wise cp.async (rows that are not 16-byte multiples,
+                                 boxes wider than 256) or global loads (naive) */
     int64_t points;           /* interior points updated per time step (global grid) */
     char kernel_name[128];    /* lowered name of the main kernel */
     int32_t reg_split[2];     /* warp-specialised ST_TB_RT kernel: registers per thread of the
@@ -370,9 +374,11 @@ int stencil_run_group(stencil_plan_t *plans, int nplans, const void *const *ins,
  *         and flag words, mapped into this process (stencil_ipc_open_handle, or
  *         plain pointers for plans of one process);
  *   flags 16 bytes of device memory per rank (flags[0] is written by rank-1,
- *         flags[1] by rank+1), zeroed by the caller before any rank registers;
- *         one flag buffer serves every plan of the rank (epochs are counted
- *         per flag buffer, so all ranks must run the same sequence of runs);
+ *         flags[1] by rank+1, flags[2] is the rank's own epoch counter, kept
+ *         on the device), zeroed by the caller before any rank registers; one
+ *         flag buffer serves every plan of the rank (epochs are counted per
+ *         flag buffer, so all ranks must run the same sequence of runs; a new,
+ *         zeroed buffer starts a new count);
  *   owned_planes  the rank's dims[0].
  * Slab layout, ghost depth and edge/interior split as stencil_plan_set_comm.
  * stencil_oc_sweep needs an NCCL communicator (E_STATE with this transport). */

@@ -84,11 +84,18 @@ __global__ void k_fill(T* __restrict__ dst, long long bz, long long by, long lon
 }
 
 // P2P transport (fused halo): publish / await an epoch in neighbours' flag
-// words. The signal runs after the edge kernels in stream order; its
-// system-scope fence + release store makes their peer stores visible before
-// the flag. The wait spins on acquire loads (one thread, sleeping between
-// polls) so that later kernels on the stream see the neighbours' planes.
-__global__ void k_p2p_signal(unsigned* a, unsigned* b, unsigned v) {
+// words. The rank's own epoch counter lives in its flag buffer (word 2, zeroed
+// with the buffer), so a new buffer always starts a new count -- a host-side
+// counter keyed by address would outlive a freed buffer whose address the
+// allocator hands out again, and the ranks would wait for different epochs.
+// The signal runs after the edge kernels in stream order: it advances the
+// counter, then a system-scope fence + release store makes the edge kernels'
+// peer stores visible before the flag. The wait spins on acquire loads (one
+// thread, sleeping between polls) until both neighbours reached the rank's
+// current epoch, so later kernels on the stream see their planes.
+__global__ void k_p2p_signal(unsigned* a, unsigned* b, unsigned* ctr) {
+  const unsigned v = *ctr + 1;
+  *ctr = v;
   __threadfence_system();
   if (a) asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(a), "r"(v) : "memory");
   if (b) asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(b), "r"(v) : "memory");
@@ -100,7 +107,8 @@ __device__ __forceinline__ unsigned ld_acquire_sys(const unsigned* p) {
   return v;
 }
 
-__global__ void k_p2p_wait(const unsigned* a, const unsigned* b, unsigned v) {
+__global__ void k_p2p_wait(const unsigned* a, const unsigned* b, const unsigned* ctr) {
+  const unsigned v = *ctr;
   // epochs grow monotonically (wrap-safe comparison)
   if (a) while ((int)(ld_acquire_sys(a) - v) < 0) __nanosleep(128);
   if (b) while ((int)(ld_acquire_sys(b) - v) < 0) __nanosleep(128);
@@ -169,17 +177,17 @@ int launch_fill(void* dst, int dtype, const int64_t box[3], const int64_t org[3]
   return STENCIL_OK;
 }
 
-int launch_p2p_signal(uint32_t* a, uint32_t* b, uint32_t v, cudaStream_t s) {
+int launch_p2p_signal(uint32_t* a, uint32_t* b, uint32_t* ctr, cudaStream_t s) {
   if (!a && !b) return STENCIL_OK;
-  k_p2p_signal<<<1, 1, 0, s>>>(a, b, v);
+  k_p2p_signal<<<1, 1, 0, s>>>(a, b, ctr);
   g_launches.fetch_add(1);
   SM_CUDA(cudaGetLastError());
   return STENCIL_OK;
 }
 
-int launch_p2p_wait(const uint32_t* a, const uint32_t* b, uint32_t v, cudaStream_t s) {
+int launch_p2p_wait(const uint32_t* a, const uint32_t* b, const uint32_t* ctr, cudaStream_t s) {
   if (!a && !b) return STENCIL_OK;
-  k_p2p_wait<<<1, 1, 0, s>>>(a, b, v);
+  k_p2p_wait<<<1, 1, 0, s>>>(a, b, ctr);
   g_launches.fetch_add(1);
   SM_CUDA(cudaGetLastError());
   return STENCIL_OK;

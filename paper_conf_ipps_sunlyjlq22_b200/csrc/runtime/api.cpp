@@ -767,11 +767,10 @@ static int run_group(const std::vector<stencil_plan_s*>& Ps, const std::vector<c
       if (c->has_hi && down)
         SM_CUDA(cudaMemcpyAsync((char*)c->hi.in + (G - down) * pb, (const char*)ins[k] + (G + n - down) * pb,
                                 down * pb, cudaMemcpyDeviceToDevice, P->stream));
-      const uint32_t e = ++*p2p_epoch(c->self.flags);
-      SM_TRY(launch_p2p_signal(c->has_lo ? c->lo.flags + 1 : nullptr, c->has_hi ? c->hi.flags : nullptr, e,
-                               P->stream));
-      SM_TRY(launch_p2p_wait(c->has_lo ? c->self.flags : nullptr, c->has_hi ? c->self.flags + 1 : nullptr, e,
-                             P->stream));
+      SM_TRY(launch_p2p_signal(c->has_lo ? c->lo.flags + 1 : nullptr, c->has_hi ? c->hi.flags : nullptr,
+                               c->self.flags + 2, P->stream));
+      SM_TRY(launch_p2p_wait(c->has_lo ? c->self.flags : nullptr, c->has_hi ? c->self.flags + 1 : nullptr,
+                             c->self.flags + 2, P->stream));
       SM_TRY(launch_frame_copy(ins[k], outs[k], elem, gs[k], P->stream));
       if (launches >= 2) SM_TRY(launch_frame_copy(ins[k], P->ws, elem, gs[k], P->stream));
     }
@@ -801,7 +800,11 @@ static int run_group(const std::vector<stencil_plan_s*>& Ps, const std::vector<c
       // fused halo: edge kernels also store the planes the neighbours need
       // into their ghost planes (same parity buffer), publish, compute the
       // interior, then await the neighbours before the next launch
-      const int E = tl_next * std::max(P0->pat.zlo, P0->pat.zhi);
+      // edge depth: the planes the neighbours need next (tl_next steps) and
+      // at least what this launch's interior would otherwise read from the
+      // ghost planes (tl steps) -- those ghosts belong to the buffer the
+      // neighbours' next edge launches overwrite once they have our signal
+      const int E = std::max(tl, tl_next) * std::max(P0->pat.zlo, P0->pat.zhi);
       const bool to_out = (launches - 1 - i) % 2 == 0;
       for (size_t k = 0; k < np; ++k) {
         stencil_plan_s* P = Ps[k];
@@ -825,16 +828,15 @@ static int run_group(const std::vector<stencil_plan_s*>& Ps, const std::vector<c
         } else {
           SM_TRY(launch_sweep(P, vs[k], ks[k], src[k], dst[k], g));
         }
-        const uint32_t e = ++*p2p_epoch(c->self.flags);
-        SM_TRY(launch_p2p_signal(c->has_lo ? c->lo.flags + 1 : nullptr, c->has_hi ? c->hi.flags : nullptr, e,
-                                 P->stream));
+        SM_TRY(launch_p2p_signal(c->has_lo ? c->lo.flags + 1 : nullptr, c->has_hi ? c->hi.flags : nullptr,
+                                 c->self.flags + 2, P->stream));
         GridArg gi = gs[k];
         if (gi.cz1 - gi.cz0 > 2 * E) {
           gi.cz0 += E; gi.cz1 -= E;
           SM_TRY(launch_sweep(P, vs[k], ks[k], src[k], dst[k], gi));
         }
-        SM_TRY(launch_p2p_wait(c->has_lo ? c->self.flags : nullptr, c->has_hi ? c->self.flags + 1 : nullptr, e,
-                               P->stream));
+        SM_TRY(launch_p2p_wait(c->has_lo ? c->self.flags : nullptr, c->has_hi ? c->self.flags + 1 : nullptr,
+                               c->self.flags + 2, P->stream));
       }
     } else if (slab && more) {
       // The edge planes (the ones the neighbours need next) run on a

@@ -160,11 +160,10 @@ struct Comm {
   stencil_p2p_buffers_t self{}, lo{}, hi{};
   bool has_lo = false, has_hi = false;
 };
-// P2P transport: epoch counter of a flag buffer (shared by the rank's plans)
-uint32_t* p2p_epoch(const void* flags);
-int launch_p2p_signal(uint32_t* flag_a, uint32_t* flag_b, uint32_t v, cudaStream_t s);
+// P2P transport: word 2 of a rank's flag buffer is its epoch counter (device)
+int launch_p2p_signal(uint32_t* flag_a, uint32_t* flag_b, uint32_t* ctr, cudaStream_t s);
 int launch_fma_probe(int dtype, long long iters, int blocks_per_sm, void* sink, double* flops, cudaStream_t s);
-int launch_p2p_wait(const uint32_t* flag_a, const uint32_t* flag_b, uint32_t v, cudaStream_t s);
+int launch_p2p_wait(const uint32_t* flag_a, const uint32_t* flag_b, const uint32_t* ctr, cudaStream_t s);
 void comm_destroy(Comm* c);
 int comm_create_stream_events(Comm* c);
 // Halo plane ranges (local plane indices) of a launch fusing `tl` steps.

@@ -4,23 +4,12 @@
 // planes (peer memory, see smart::Grid::peer_lo/peer_hi in the kernels) and a
 // one-thread kernel publishes an epoch in the neighbour's flag word; the
 // neighbour's next edge kernels wait for it (run_group in api.cpp). This file
-// holds registration, the per-flag-buffer epoch counters and CUDA IPC.
+// holds registration and CUDA IPC; the epoch counter is word 2 of the flag buffer.
 #include <cstring>
 #include <map>
 #include <mutex>
 
 #include "internal.h"
-
-namespace smart_rt {
-
-uint32_t* p2p_epoch(const void* flags) {
-  static std::mutex mu;
-  static std::map<const void*, uint32_t> epochs;
-  std::lock_guard<std::mutex> lk(mu);
-  return &epochs[flags];   // std::map nodes are stable
-}
-
-}  // namespace smart_rt
 
 using namespace smart_rt;
 
