@@ -417,11 +417,13 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   o << "  static constexpr int TMID = " << tmid << ";\n";
   o << "  static constexpr int MVX = " << (v.midvx > 0 ? v.midvx : std::max(v.vx, 1)) << ";\n";
   o << "  static constexpr bool SPLITMID = " << (v.splitmid ? "true" : "false") << ";\n";
-  {   // k_stream_tb_rt hand-off details (dev overrides for A/B measurements)
+  {   // k_stream_tb_rt hand-off details, off by default: measured on C2 (same box,
+      // 2 runs each) elected-lane arrivals 552 -> 546 GStencil/s, warp-aligned
+      // stage-1 tiles 552 -> 530, both 528 (dev overrides for A/B measurements)
     const char* el = getenv("STENCIL_ELECT");
     const char* wa = getenv("STENCIL_WALIGN");
-    o << "  static constexpr bool ELECT = " << ((el ? atoi(el) : 1) ? "true" : "false") << ";\n";
-    o << "  static constexpr bool WALIGN = " << ((wa ? atoi(wa) : 1) ? "true" : "false") << ";\n";
+    o << "  static constexpr bool ELECT = " << ((el ? atoi(el) : 0) ? "true" : "false") << ";\n";
+    o << "  static constexpr bool WALIGN = " << ((wa ? atoi(wa) : 0) ? "true" : "false") << ";\n";
   }
   o << "  static constexpr bool XM = " << (v.xm ? "true" : "false") << ";   // merge along x (2-D streaming)\n";
   o << "  static constexpr bool TMA = " << (v.tma ? "true" : "false") << ";   // streaming TB staging (else cp.async)\n";

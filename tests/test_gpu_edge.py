@@ -18,6 +18,7 @@ Grids are ragged against every tile, and both 16-byte-aligned rows (TMA staging)
 and unaligned rows (cp.async staging of the streaming TB kernels) are covered.
 """
 import concurrent.futures as cf
+import os
 
 import numpy as np
 import pytest
@@ -35,7 +36,7 @@ MIXED = {"mixed3d", "mixed3d_r2", "mixed2d"}
 def _plans(acc, c, dims, dtype, ocs, params=None):
     def mk(oc):
         return sm.Plan(dims, acc, c, dtype, oc, params(oc) if callable(params) else params)
-    with cf.ThreadPoolExecutor(8) as ex:
+    with cf.ThreadPoolExecutor(os.cpu_count() or 8) as ex:
         return dict(zip(ocs, ex.map(mk, ocs)))
 
 
@@ -126,7 +127,7 @@ def test_label_pass_settings(gpu, name, dims, dtype):
             except sm.StencilError as e:
                 assert e.code == -3, (sm.oc_name(oc), k, str(e))
                 return None
-        with cf.ThreadPoolExecutor(8) as ex:
+        with cf.ThreadPoolExecutor(os.cpu_count() or 8) as ex:
             plans = dict(zip(sm.oc_list(), ex.map(mk, sm.oc_list())))
         for oc, p in plans.items():
             if p is None:

@@ -42,7 +42,7 @@ def _plans(acc, c, dims, dtype, ocs, params=None):
             if e.code == -3:
                 return None
             raise
-    with cf.ThreadPoolExecutor(8) as ex:
+    with cf.ThreadPoolExecutor(os.cpu_count() or 8) as ex:
         return dict(zip(ocs, ex.map(mk, ocs)))
 
 
