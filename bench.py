@@ -395,8 +395,8 @@ def measure_fma_peak(sm, dtype: str, local: int, seconds: float = 2.0) -> dict:
     c = clk.result()
     return {"sustained": round(statistics.median(half), 2), "burst": round(max(vals), 2), "unit": "TFLOP/s",
             "dtype": dtype, "launches": len(vals), "sm_mhz": c["sm_mhz"], "reasons": c["reasons"],
-            "how": "stencil_fma_probe: 148 SMs x 8 CTAs x 256 threads, 8 independent FMA chains per thread, "
-                   "~20 ms launches back to back; 2 flops per FMA"}
+            "how": "stencil_fma_probe: 148 SMs x 8 CTAs x 256 threads, 12 independent FMA chains per thread with "
+                   "immediate operands, ~20 ms launches back to back; 2 flops per FMA"}
 
 
 def _roofline(name, sm, pinfo, oc, pts, steps, kern_ms, kern_n, total_ms, nsteps_timed, elem, dtype, peak, peak_kind,

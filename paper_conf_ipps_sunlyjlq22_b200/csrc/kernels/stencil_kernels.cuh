@@ -239,22 +239,35 @@ struct SmemPlane {                    // shared memory, compile-time row pitch
 };
 
 // Even/odd-split rows (k_stream_tb_rt, S::SPLITMID; fp64, VX = 2): column c of
-// a row lives at (c & 1) * LX/2 + (c >> 1). A thread's x-neighbour columns then
-// come from contiguous 8-byte loads (the odd array for c - 1, the even one for
-// c + 2) instead of 8-byte halves of 16-byte vectors at a 16-byte stride, which
-// cost a 16-byte vector's shared-memory wavefronts for half the data.
-template <class T, int LX>
+// a row lives at (c & 1) * SO + (c >> 1), rows SP elements apart. A thread's
+// x-neighbour columns then come from contiguous 8-byte loads (the odd array for
+// c - 1, the even one for c + 2) instead of 8-byte halves of 16-byte vectors at
+// a 16-byte stride, which cost a 16-byte vector's shared-memory wavefronts for
+// half the data. The odd array's offset SO is chosen so that a half-warp phase
+// of 8-byte stores from 16 consecutive columns c0.. puts its 8 even and 8 odd
+// values on disjoint banks: the odd block starts SO - (c0 & 1) elements after
+// the even one, which must be 64 bytes past a multiple of 128, i.e. SO = 8 +
+// (c0 & 1) (mod 16) for fp64; c0's parity is the same for every phase that lies
+// within one tile row (K below). With SO = LX/2 = 34 the two halves overlapped
+// on up to 14 banks: 17 M of C2's 24 M bank-conflict wavefronts per launch.
+template <class T, int SP, int SO>
 struct SplitPlane {
   const T* p;                          // even array of row 0 at the thread's first output vector
   __device__ __forceinline__ void get(int j, int kv, T (&w)[2]) const {
-    w[0] = p[j * LX + kv];
-    w[1] = p[j * LX + LX / 2 + kv];
+    w[0] = p[j * SP + kv];
+    w[1] = p[j * SP + SO + kv];
   }
 };
-template <int LX>
+template <int SP, int SO>
 __device__ __forceinline__ int split_idx(int row, int col) {
-  return row * LX + (col & 1) * (LX / 2) + (col >> 1);
+  return row * SP + (col & 1) * SO + (col >> 1);
 }
+// odd-array offset >= lx / 2, == 8 + (k & 1) (mod 16), k = column parity of the
+// stores' phases; and the row pitch
+__host__ __device__ constexpr int split_off(int lx, int k) {
+  return lx / 2 + ((8 + (k & 1) - (lx / 2) % 16) + 32) % 16;
+}
+__host__ __device__ constexpr int split_pitch(int lx, int k) { return split_off(lx, k) + lx / 2 + 1; }
 
 template <class T, int VX, int NROW>
 struct GlobalPlane {                  // global memory through the read-only path
@@ -1191,7 +1204,12 @@ struct StreamTbRtCfg {
   static __device__ __forceinline__ constexpr int xoff(int s) { return S::XSHIFT ? (TT - s) * S::XLO : XOFF; }
   static constexpr int LX = ((XOFF + BX + TT * S::XHI + ALN - 1) / ALN) * ALN;
   static constexpr int LY = BY * TG::MY + TT * (S::YLO + S::YHI);
-  static constexpr int PLANE = ((LX * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
+  // even/odd-split last ring (S::SPLITMID; only without XSHIFT): its own row
+  // pitch SP, odd arrays at SO; K = ring column of stage TT-1's tile column 0
+  static constexpr int MVS = S::MVX;
+  static constexpr int K = XOFF - ((S::XLO + MVS - 1) / MVS) * MVS;
+  static constexpr int SO = split_off(LX, K), SP = S::SPLITMID ? split_pitch(LX, K) : LX;
+  static constexpr int PLANE = (((SP > LX ? SP : LX) * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
   static constexpr int MI = S::MI;
   static constexpr int PADF = 128 / (int)sizeof(T);
   static constexpr int PADB = ((MI * LX + ALN) * (int)sizeof(T) + 127) / 128 * 128 / (int)sizeof(T);
@@ -1373,7 +1391,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
             if (rows & (1u << m)) {
               if constexpr (SPL) {
 #pragma unroll
-                for (int v = 0; v < MV; ++v) dst[split_idx<C::LX>(lrow + m, lcol + v)] = res[m][v];
+                for (int v = 0; v < MV; ++v) dst[split_idx<C::SP, C::SO>(lrow + m, lcol + v)] = res[m][v];
               } else {
                 stg_vec<T, MV>(dst + lb + m * C::LX, res[m]);
               }
@@ -1394,7 +1412,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
                 if (gx < 0 || gx >= g.nx || gx - xb + XO_W >= C::LX) continue;
                 const bool upd = rowupd && gx >= g.ux0 && gx < g.ux1;
                 const T val = upd ? res[m][v] : (s == 1 ? fr[m * C::LX + v] : __ldg(frame + gx));
-                if constexpr (SPL) dst[split_idx<C::LX>(lrow + m, lcol + v)] = val;
+                if constexpr (SPL) dst[split_idx<C::SP, C::SO>(lrow + m, lcol + v)] = val;
                 else d[v] = val;
               }
             }
@@ -1437,7 +1455,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         if (act) {
           const T* pm = mid + (MR * (TT - 2) + si) * C::PLANE;
           if constexpr (S::SPLITMID) {
-            SplitPlane<T, C::LX> pl{pm + row0 * C::LX + (col0 >> 1)};
+            SplitPlane<T, C::SP, C::SO> pl{pm + row0 * C::SP + (col0 >> 1)};
             run_scatter<S, VX, M, U>(pl, acc);
           } else {
             SmemPlane<T, VX, C::LX> pl{pm + row0 * C::LX + col0};
