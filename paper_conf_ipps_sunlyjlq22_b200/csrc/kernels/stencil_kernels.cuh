@@ -1173,7 +1173,10 @@ struct TbRtStage {
   static constexpr int NTX = (TXL + BX + HX1 + VXM - 1) / VXM;
   static constexpr int RY = BY * MY + HY0 + HY1;
   static constexpr int NTY = (RY + MI - 1) / MI;
-  static constexpr int NT = NTX * NTY;
+  // S::WALIGN == 2: tile rows padded to whole half-warps (idle lanes), so no
+  // 16-lane phase of a shared-memory access spans two tile rows
+  static constexpr int NTXP = S::WALIGN == 2 ? (NTX + 15) / 16 * 16 : NTX;
+  static constexpr int NT = NTXP * NTY;
   static constexpr int W = (NT + 31) / 32;                 // warps of group s
 };
 
@@ -1324,15 +1327,16 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     constexpr int MV = G::VXM;
     constexpr bool XOVER = XO_W - G::TXL + G::NTX * MV > C::LX;
     const int t = tid - 32 * W0;
-    const bool act = t < G::NT;
+    bool act = t < G::NT;
     // tile (column cx, row cy) of thread t. S::WALIGN: the first NXM columns of
     // every tile row (a multiple of 32) are whole warps of one tile row, the
     // remaining NTX - NXM columns of all rows go to the last warp(s); otherwise
     // row-major over NTX columns, where a warp straddling two tile rows hits
     // the same banks twice (a third shared-memory wavefront per access)
-    constexpr int NXM = S::WALIGN ? (G::NTX / 32) * 32 : 0, NXE = G::NTX - NXM;
+    constexpr int NXM = S::WALIGN == 1 ? (G::NTX / 32) * 32 : 0, NXE = G::NTXP - NXM;
     const int cx = t < NXM * G::NTY ? t % (NXM ? NXM : 1) : NXM + (t - NXM * G::NTY) % NXE;
     const int cy = t < NXM * G::NTY ? t / (NXM ? NXM : 1) : (t - NXM * G::NTY) / NXE;
+    if (cx >= G::NTX) act = false;                              // (WALIGN == 2 padding lanes)
     const int gx0 = xb - G::TXL + cx * MV;
     const int gy0 = yb - G::HY0 + cy * MI;
     const int lb_r = (gy0 - Y0) * C::LX + (gx0 - xb + XO_R);   // tile origin in the source ring

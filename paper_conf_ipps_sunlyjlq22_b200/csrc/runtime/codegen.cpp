@@ -177,7 +177,9 @@ int Variant::tbrt_threads(const Pattern& p, int elem, int* wl_out) const {
     const int hy0 = (tt - s) * p.ylo, hy1 = (tt - s) * p.yhi;
     const int mvx = midvx > 0 ? midvx : vx;
     const int txl = xshift ? hx0 : roundup(hx0, mvx);
-    const int ntx = (txl + bx + hx1 + mvx - 1) / mvx;
+    int ntx = (txl + bx + hx1 + mvx - 1) / mvx;
+    if (const char* wa = getenv("STENCIL_WALIGN"))   // dev: padded tile rows (TbRtStage::NTXP)
+      if (atoi(wa) == 2) ntx = roundup(ntx, 16);
     const int nty = (rows() + hy0 + hy1 + mi - 1) / mi;
     warps += (ntx * nty + 31) / 32;
   }
@@ -427,7 +429,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
     const char* el = getenv("STENCIL_ELECT");
     const char* wa = getenv("STENCIL_WALIGN");
     o << "  static constexpr bool ELECT = " << ((el ? atoi(el) : 0) ? "true" : "false") << ";\n";
-    o << "  static constexpr bool WALIGN = " << ((wa ? atoi(wa) : 0) ? "true" : "false") << ";\n";
+    o << "  static constexpr int WALIGN = " << (wa ? atoi(wa) : 0) << ";\n";
   }
   o << "  static constexpr bool XM = " << (v.xm ? "true" : "false") << ";   // merge along x (2-D streaming)\n";
   o << "  static constexpr bool TMA = " << (v.tma ? "true" : "false") << ";   // streaming TB staging (else cp.async)\n";
