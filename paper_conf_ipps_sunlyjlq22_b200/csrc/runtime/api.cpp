@@ -141,7 +141,10 @@ static void default_params(uint32_t oc, int ndim, int dtype, stencil_params_t* p
     // 64 x 32-row output tiles (8 threads x merge 4 rows), 3 planes in flight
     p->vx = vmax; p->bx = 32 * vmax; p->by = 8; p->bz = 1;
     if (merge) p->merge = 4;
-    if (oc & STENCIL_OC_PR) p->pr_stages = 3;
+    // 4 planes in flight: the stage-1 warps waited on the input ring for 23% of
+    // their ncu stall samples with 3 (round 2, C2 same box: 563 -> 585 GStencil/s
+    // with 4; 6: 585; 8 no longer fits one CTA per SM)
+    if (oc & STENCIL_OC_PR) p->pr_stages = 4;
   } else {
     p->vx = vmax; p->bx = 32 * vmax; p->by = merge ? 4 : 8; p->bz = 1;
   }
