@@ -11,7 +11,7 @@ out=gpurun_out/sanitize_summary.txt
 for tool in ${TOOLS:-memcheck racecheck synccheck}; do
   for c in ${CASES:-naive tiled_tb stream_gather stream_rt stream_cpasync stream_tb tbrt_split tbrt_xshift tbrt_cpasync tbrt_t3_fp32 xmerge_2d tbrt_2d p2p}; do
     log=gpurun_out/san_${tool}_${c}.log
-    timeout 600 compute-sanitizer --tool $tool --print-limit 20 --error-exitcode 99 \
+    timeout 300 compute-sanitizer --tool $tool --print-limit 20 --error-exitcode 99 \
         python scripts/sanitize_case.py $c > $log 2>&1
     rc=$?
     summ=$(grep -E "ERROR SUMMARY|RACECHECK SUMMARY|max rel err" $log | tr '\n' ' ')
