@@ -381,6 +381,9 @@ int stencil_run_group(stencil_plan_t *plans, int nplans, const void *const *ins,
  *         zeroed buffer starts a new count);
  *   owned_planes  the rank's dims[0].
  * Slab layout, ghost depth and edge/interior split as stencil_plan_set_comm.
+ * Registration also compiles and loads every kernel a run can launch (the main
+ * one and the TB remainder kernels), so that no module load happens once ranks
+ * sharing a device wait on each other's flags.
  * stencil_oc_sweep needs an NCCL communicator (E_STATE with this transport). */
 typedef struct {
     void *in, *out, *ws;

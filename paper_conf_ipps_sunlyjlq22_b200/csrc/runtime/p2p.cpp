@@ -15,6 +15,7 @@ using namespace smart_rt;
 
 namespace smart_rt {
 int slab_setup_ext(stencil_plan_s* P, int rank, int nranks, int transport);
+int preload_kernels(stencil_plan_s* P);
 }
 
 static bool bufs_ok(const stencil_p2p_buffers_t* b) { return b && b->in && b->out && b->flags && b->owned_planes > 0; }
@@ -42,7 +43,8 @@ extern "C" int stencil_plan_set_p2p(stencil_plan_t P, int rank, int nranks, cons
   c->self = *self;
   if (lo) { c->lo = *lo; c->has_lo = true; }
   if (hi) { c->hi = *hi; c->has_hi = true; }
-  return STENCIL_OK;
+  // every kernel loaded before any run enqueues a flag wait (preload_kernels)
+  return preload_kernels(P);
 }
 
 extern "C" int stencil_ipc_get_handle(const void* dev_ptr, uint8_t* handle, int64_t* offset) {
