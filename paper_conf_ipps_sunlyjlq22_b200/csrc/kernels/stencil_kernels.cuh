@@ -1295,22 +1295,38 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
   if (warp == 0) {
     if constexpr (S::TMA) {
       if (tid == 0) {
+        int slot = 0;
+        unsigned ph = 0;                                 // (j / NR) & 1
 #pragma unroll 1
         for (int j = 0; j < nin; ++j) {
-          const int slot = j % NR;
-          if (j >= NR) mbar_wait_sleep(&empty_in[slot], (unsigned)((j / NR - 1) & 1));
+          if (j >= NR) mbar_wait_sleep(&empty_in[slot], ph ^ 1u);
           mbar_expect_tx(&full_in[slot], C::LX * C::LY * (unsigned)sizeof(T));
           tma_load_3d(ring0 + slot * C::PLANE, &tmap, &full_in[slot], X0, Y0, pin0 + j);
+          if (++slot == NR) { slot = 0; ph ^= 1u; }
         }
       }
-    } else {   // rows not TMA-aligned: the whole warp stages planes with cp.async
+    } else {
+      // rows not TMA-aligned: the whole warp stages planes with cp.async, one
+      // commit group per plane, NS planes in flight; plane j - (NS-1) is
+      // published (a plain release-arrive by every lane) once cp.async.wait_group
+      // says its group has landed -- the classic multistage cp.async pipeline
+      // (compute-sanitizer racecheck flagged the variant that published with
+      // cp.async.mbarrier.arrive.noinc; this form is clean)
+      int slot = 0;
+      unsigned ph = 0;
 #pragma unroll 1
       for (int j = 0; j < nin; ++j) {
-        const int slot = j % NR;
-        if (j >= NR) mbar_wait_sleep(&empty_in[slot], (unsigned)((j / NR - 1) & 1));
+        if (j >= NR) mbar_wait_sleep(&empty_in[slot], ph ^ 1u);
         stage_plane_cp_async<T, C::LX, C::LY, 32>(ring0 + slot * C::PLANE, in, g, X0, Y0, pin0 + j, tid);
-        cp_async_mbar_arrive(&full_in[slot]);
+        cp_async_commit();
+        if (j >= NS - 1) {
+          cp_async_wait<NS - 1>();
+          mbar_arrive(&full_in[(j - (NS - 1)) % NR]);
+        }
+        if (++slot == NR) { slot = 0; ph ^= 1u; }
       }
+      cp_async_wait<0>();
+      for (int j = nin - (NS - 1) > 0 ? nin - (NS - 1) : 0; j < nin; ++j) mbar_arrive(&full_in[j % NR]);
     }
     return;
   }
@@ -1364,27 +1380,30 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     // NZ unrolled plane bodies (compile-time queue rotation), or one body and
     // a register shift of the queue for large op tables (S::RTSHIFT)
     constexpr int UNR = S::RTSHIFT ? 1 : NZ;
+    // ring slots and mbarrier phases advance incrementally (the input ring has
+    // NS + ZHI slots, generally not a power of two: j % NR and j / NR per plane
+    // cost a dozen integer instructions on every stage warp's critical path)
+    int si = 0, so = 0, sf = (NR - S::ZHI % NR) % NR;   // slots of planes j, j (own ring), j - ZHI
+    unsigned pin = 0, pout = 0;                          // phases (j / DIN) & 1, (j / MR) & 1
 #pragma unroll 1
     for (int jb = 0; jb < nin; jb += UNR) {
       static_for<0, UNR>([&](auto ic) {
         constexpr int U = S::RTSHIFT ? NZ - 1 : decltype(ic)::value;
         const int j = jb + decltype(ic)::value;
         if (j >= nin) return;
-        const int si = j % DIN;
         const T* src = s == 1 ? ring0 + si * C::PLANE : mid + (MR * (s - 2) + si) * C::PLANE;
-        mbar_wait_sleep(&fin[si], (unsigned)((j / DIN) & 1));
+        mbar_wait_sleep(&fin[si], pin);
         if constexpr (!S::RTSHIFT) zero_acc<T, MV, MI>(acc[U]);   // a new output plane starts
         if (act) {
           SmemPlane<T, MV, C::LX> pl{src + lb_r - S::XSH};
           run_scatter_ops<S, typename S::Mid, MV, MI, U>(pl, acc);
         }
         if (s > 1) warp_arrive<S::ELECT>(&ein[si]);      // input slot read (stage 1: below)
-        const int so = j % MR;
         T* dst = mid + (MR * (s - 1) + so) * C::PLANE;
-        if (j >= MR) mbar_wait_sleep(&empty_s(s)[so], (unsigned)((j / MR - 1) & 1));
+        if (j >= MR) mbar_wait_sleep(&empty_s(s)[so], pout ^ 1u);
         const int zo = pin0 + j - s * S::ZHI;            // plane completed now
         // stage 1: input plane zo (= index j - ZHI) is still in the ring
-        const T* fr = ring0 + ((j - S::ZHI + NR) % NR) * C::PLANE + lb_r;
+        const T* fr = ring0 + sf * C::PLANE + lb_r;
         const bool zin = zo >= 0 && zo < g.nz;
         const bool zupd = zo >= g.uz0 && zo < g.uz1;
         const T(&res)[MI][MV] = acc[(U + 1) % NZ];
@@ -1422,9 +1441,12 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
             }
           }
         }
-        if (s == 1 && j >= S::ZHI) warp_arrive<S::ELECT>(&ein[(j - S::ZHI) % NR]);   // frame source released
+        if (s == 1 && j >= S::ZHI) warp_arrive<S::ELECT>(&ein[sf]);   // frame source released
         warp_arrive<S::ELECT>(&full_s(s)[so]);           // stage-s plane written
         if constexpr (S::RTSHIFT) shift_queue<T, NZ, MI, MV>(acc);
+        if (++si == DIN) { si = 0; pin ^= 1u; }
+        if (++so == MR) { so = 0; pout ^= 1u; }
+        if (++sf == NR) sf = 0;
       });
     }
   });

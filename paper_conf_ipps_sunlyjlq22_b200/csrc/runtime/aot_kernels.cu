@@ -196,6 +196,20 @@ int launch_p2p_wait(const uint32_t* a, const uint32_t* b, const uint32_t* ctr, c
   return STENCIL_OK;
 }
 
+// Force-load the pattern-independent kernels a slab run launches. With CUDA's
+// lazy module loading a kernel is loaded at its first launch, and that load can
+// wait on the context; several P2P slab plans of one process enqueue spinning
+// k_p2p_wait kernels on their streams, so a first k_frame_copy launch behind one
+// of them deadlocked (found by the sanitizer pass's in-process P2P case).
+int preload_aot_kernels() {
+  cudaFuncAttributes a;
+  SM_CUDA(cudaFuncGetAttributes(&a, k_frame_copy<unsigned long long>));
+  SM_CUDA(cudaFuncGetAttributes(&a, k_frame_copy<unsigned>));
+  SM_CUDA(cudaFuncGetAttributes(&a, k_p2p_signal));
+  SM_CUDA(cudaFuncGetAttributes(&a, k_p2p_wait));
+  return STENCIL_OK;
+}
+
 int launch_fma_probe(int dtype, long long iters, int blocks_per_sm, void* sink, double* flops, cudaStream_t s) {
   int dev = 0, nsm = 0;
   SM_CUDA(cudaGetDevice(&dev));

@@ -632,12 +632,14 @@ static int get_tb_rem_kernel(stencil_plan_s* P, int tt, Variant* vout, Kernel* k
 int run_device(stencil_plan_s* P, const void* in, void* out, int steps);
 
 // Compile and load every kernel a run of this plan can launch (the main one and
-// the TB remainder kernels of depth 1..T-1) now. P2P registration calls it:
+// the TB remainder kernels of depth 1..T-1, and the AOT frame-copy / flag
+// kernels, which CUDA loads lazily at first launch) now. P2P registration calls it:
 // several slab plans of ONE process (one GPU) enqueue spin-waiting flag kernels
 // on their streams, and a module load inside a later plan's first run could then
 // wait on the context behind a spin that only that run would release (seen as a
 // hang of two in-process slabs whose kernels had not been loaded before).
 int preload_kernels(stencil_plan_s* P) {
+  SM_TRY(preload_aot_kernels());
   SM_TRY(ensure_loaded(P));
   const int T = P->var.family == FAM_TILED || P->var.family == FAM_STREAM_TB ? P->var.tt : 1;
   for (int tl = 1; tl < T; ++tl) {

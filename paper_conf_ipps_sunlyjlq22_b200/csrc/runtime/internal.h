@@ -162,6 +162,7 @@ struct Comm {
 };
 // P2P transport: word 2 of a rank's flag buffer is its epoch counter (device)
 int launch_p2p_signal(uint32_t* flag_a, uint32_t* flag_b, uint32_t* ctr, cudaStream_t s);
+int preload_aot_kernels();
 int launch_fma_probe(int dtype, long long iters, int blocks_per_sm, void* sink, double* flops, cudaStream_t s);
 int launch_p2p_wait(const uint32_t* flag_a, const uint32_t* flag_b, const uint32_t* ctr, cudaStream_t s);
 void comm_destroy(Comm* c);
