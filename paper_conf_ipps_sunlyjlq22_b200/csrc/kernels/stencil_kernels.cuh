@@ -1212,8 +1212,13 @@ struct StreamTbRtCfg {
   static constexpr int MVS = S::MVX;
   static constexpr int K = XOFF - ((S::XLO + MVS - 1) / MVS) * MVS;
   static constexpr int SO = split_off(LX, K), SP = S::SPLITMID ? split_pitch(LX, K) : LX;
-  static constexpr int PLANE = (((SP > LX ? SP : LX) * LY * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T);
   static constexpr int MI = S::MI;
+  // slot stride: the plane plus the rows a VX x MI intermediate tile of the last
+  // tile row reads past it (discarded values) -- without the gap those reads fall
+  // into the next slot while the producer refills it (a benign data race that
+  // compute-sanitizer racecheck reports on the cp.async path)
+  static constexpr int PLANE = (((SP > LX ? SP : LX) * LY + MI * LX + ALN) * (int)sizeof(T) + 127) / 128 * 128 /
+                               (int)sizeof(T);
   static constexpr int PADF = 128 / (int)sizeof(T);
   static constexpr int PADB = ((MI * LX + ALN) * (int)sizeof(T) + 127) / 128 * 128 / (int)sizeof(T);
   static constexpr int NR = NS + S::ZHI;                     // input ring slots
@@ -1321,11 +1326,13 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         cp_async_commit();
         if (j >= NS - 1) {
           cp_async_wait<NS - 1>();
+          __threadfence_block();                         // landed copies ordered before the release
           mbar_arrive(&full_in[(j - (NS - 1)) % NR]);
         }
         if (++slot == NR) { slot = 0; ph ^= 1u; }
       }
       cp_async_wait<0>();
+      __threadfence_block();
       for (int j = nin - (NS - 1) > 0 ? nin - (NS - 1) : 0; j < nin; ++j) mbar_arrive(&full_in[j % NR]);
     }
     return;

@@ -219,7 +219,7 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     const int mv = midvx > 0 ? midvx : vx;
     const int k = xoff - roundup(p.xlo, mv);
     const int so = lx / 2 + ((8 + (k & 1) - (lx / 2) % 16) + 32) % 16, sp = splitmid ? so + lx / 2 + 1 : lx;
-    const int plane = roundup(std::max(lx, sp) * ly * elem, 128) / elem;
+    const int plane = roundup((std::max(lx, sp) * ly + mid_rows(p, elem) * lx + aln) * elem, 128) / elem;
     const int padf = 128 / elem;
     const int padb = roundup((mid_rows(p, elem) * lx + aln) * elem, 128) / elem;
     const int nr = ns + p.zhi, mr = mid_slots();
