@@ -117,7 +117,7 @@ class ClockSampler:
                         self.reasons.add(k)
             except Exception:
                 pass
-            self._stop.wait(0.02)
+            self._stop.wait(0.005)
 
     def __enter__(self):
         if self.nv:
@@ -534,6 +534,36 @@ def run_impl(args):
             }
             if math.isfinite(t) and t < best_t:
                 best_oc, best_t, best_p = oc, t, p
+        # spatial tiling reported as its own entry (shared memory is a
+        # Boolean parameter of base / BM / CM; the label pass draws it among the
+        # sampled settings, so per_oc above may hold either form): the smem = 1
+        # form of each, default tiles, median of 3 timed runs
+        if args.tiling and args.settings > 0 and len(ocs) > 1:
+            for oc in (0, sm.OC_BM, sm.OC_CM):
+                if oc not in ocs:
+                    continue
+                key = sm.oc_name(oc) + "+tiling(smem=1)"
+                try:
+                    tp = make_plan(it["acc"], it["c"], oc, {"smem": 1})
+                    tp.use_workspace(ws)
+                    tp.run(x, y, steps)
+                    ts = []
+                    for _ in range(3):
+                        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                        a.record(stream)
+                        tp.run(x, y, steps)
+                        b.record(stream)
+                        b.synchronize()
+                        ts.append(a.elapsed_time(b))
+                    t = statistics.median(ts)
+                    gs = sm.gstencil_per_s(it["points"], steps, t)
+                    per_oc[key] = {"ms": round(t, 4), "gstencil_s": round(gs, 2), "time_steps_per_launch": 1,
+                                   "hbm_frac_of_measured": round(gs * 2 * elem / peak, 4),
+                                   "hbm_frac_of_spec": round(gs * 2 * elem / HBM_SPEC_GBS, 4), "infeasible": False,
+                                   "kernel": tp.info["kernel_name"][:40]}
+                    del tp
+                except sm.StencilError as e:
+                    per_oc[key] = {"ms": None, "gstencil_s": None, "infeasible": True, "why": str(e)[:120]}
         if best_oc is None:
             best_oc, best_p = ocs[0], None
         if args.params:
@@ -723,6 +753,8 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-tiling", dest="tiling", action="store_false",
+                    help="skip the extra smem = 1 (spatial tiling) timings of base / BM / CM in per_oc")
     ap.add_argument("--slab", action="store_true", help="use the NCCL slab path even at N = 1")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p"],
                     help="halo exchange of the timed slab runs: NCCL send/recv on a comm stream, or the fused "
