@@ -1169,8 +1169,19 @@ struct TbRtStage {
   // columns, so every shared-memory access of the stage is a contiguous 8-byte
   // warp access instead of 16-byte vectors with half-used neighbours)
   static constexpr int VXM = S::MVX;
-  static constexpr int TXL = S::XSHIFT ? HX0 : ((HX0 + VXM - 1) / VXM) * VXM;
-  static constexpr int NTX = (TXL + BX + HX1 + VXM - 1) / VXM;
+  // S::FULLW (scalar columns, rounded geometry): the stage's tiles span every
+  // column of the ring rows (pitch LXF, the TMA box width), so thread t reads
+  // ring word t + const for each window element and no 16-lane phase of a load
+  // can put two tile rows on the same banks (row-straddling phases of 66-column
+  // tile rows in a 68-element pitch replayed up to 2 wavefronts each). The
+  // extra columns are computed from don't-care neighbours and never feed a
+  // valid output.
+  static constexpr bool FULLW = S::FULLW && !S::XSHIFT && VXM == 1;
+  static constexpr int ALNF = (16 / (int)sizeof(typename S::T)) > VX ? (16 / (int)sizeof(typename S::T)) : VX;
+  static constexpr int XOFFF = ((TT * S::XLO + ALNF - 1) / ALNF) * ALNF;
+  static constexpr int LXF = ((XOFFF + BX + TT * S::XHI + ALNF - 1) / ALNF) * ALNF;
+  static constexpr int TXL = FULLW ? XOFFF : S::XSHIFT ? HX0 : ((HX0 + VXM - 1) / VXM) * VXM;
+  static constexpr int NTX = FULLW ? LXF : (TXL + BX + HX1 + VXM - 1) / VXM;
   static constexpr int RY = BY * MY + HY0 + HY1;
   static constexpr int NTY = (RY + MI - 1) / MI;
   // S::WALIGN == 2: tile rows padded to whole half-warps (idle lanes), so no
@@ -1211,7 +1222,12 @@ struct StreamTbRtCfg {
   // pitch SP, odd arrays at SO; K = ring column of stage TT-1's tile column 0
   static constexpr int MVS = S::MVX;
   static constexpr int K = XOFF - ((S::XLO + MVS - 1) / MVS) * MVS;
-  static constexpr int SO = split_off(LX, K), SP = S::SPLITMID ? split_pitch(LX, K) : LX;
+  // FULLW: a phase may span two tile rows, so rows must continue each other's
+  // banks (SP = LX/2 mod 16) besides the even/odd halves (SO = 8 mod 16, the
+  // phases start on even columns)
+  static constexpr bool FW = S::FULLW && !S::XSHIFT && MVS == 1;
+  static constexpr int SO = split_off(LX, FW ? 0 : K);
+  static constexpr int SP = !S::SPLITMID ? LX : FW ? SO + LX / 2 + (16 - SO % 16) % 16 : split_pitch(LX, K);
   static constexpr int MI = S::MI;
   // slot stride: the plane plus the rows a VX x MI intermediate tile of the last
   // tile row reads past it (discarded values) -- without the gap those reads fall

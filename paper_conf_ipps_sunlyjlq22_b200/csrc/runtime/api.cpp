@@ -357,6 +357,11 @@ static int resolve_variant(stencil_plan_s* P) {
     }
     if (const char* mv = getenv("STENCIL_MID_VX"))   // dev override: intermediate-step columns per thread
       if (!v.xshift) v.midvx = std::max(0, std::min(v.vx, atoi(mv)));
+    // scalar-column stage tiles over whole ring rows (TbRtStage::FULLW)
+    v.fullw = false;
+    if (const char* fw = getenv("STENCIL_FULLW")) v.fullw = atoi(fw) != 0;   // dev override
+    if (v.midvx != 1 || v.xshift) v.fullw = false;
+    if (v.fullw && v.tbrt_threads(P->pat, elem) > 1024) v.fullw = false;
     choose_regsplit(&v, P->pat, elem);
     v.ws_threads = v.tbrt_threads(P->pat, elem);
   }

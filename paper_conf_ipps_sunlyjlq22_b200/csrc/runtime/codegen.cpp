@@ -178,6 +178,10 @@ int Variant::tbrt_threads(const Pattern& p, int elem, int* wl_out) const {
     const int mvx = midvx > 0 ? midvx : vx;
     const int txl = xshift ? hx0 : roundup(hx0, mvx);
     int ntx = (txl + bx + hx1 + mvx - 1) / mvx;
+    if (fullw) {                                  // TbRtStage::FULLW: the ring's whole rows
+      const int aln = std::max(16 / elem, vx);
+      ntx = roundup(roundup(tt * p.xlo, aln) + bx + tt * p.xhi, aln);
+    }
     if (const char* wa = getenv("STENCIL_WALIGN"))   // dev: padded tile rows (TbRtStage::NTXP)
       if (atoi(wa) == 2) ntx = roundup(ntx, 16);
     const int nty = (rows() + hy0 + hy1 + mi - 1) / mi;
@@ -218,7 +222,8 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     // even/odd-split last ring: row pitch split_pitch(lx, k) (stencil_kernels.cuh)
     const int mv = midvx > 0 ? midvx : vx;
     const int k = xoff - roundup(p.xlo, mv);
-    const int so = lx / 2 + ((8 + (k & 1) - (lx / 2) % 16) + 32) % 16, sp = splitmid ? so + lx / 2 + 1 : lx;
+    const int so = lx / 2 + ((8 + ((fullw ? 0 : k) & 1) - (lx / 2) % 16) + 32) % 16;
+    const int sp = !splitmid ? lx : fullw ? so + lx / 2 + (16 - so % 16) % 16 : so + lx / 2 + 1;
     const int plane = roundup((std::max(lx, sp) * ly + mid_rows(p, elem) * lx + aln) * elem, 128) / elem;
     const int padf = 128 / elem;
     const int padb = roundup((mid_rows(p, elem) * lx + aln) * elem, 128) / elem;
@@ -382,7 +387,23 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   // ptxas then stages them through uniform registers with LDCU + R2UR and the
   // order-2 random kernel grew from 86 to 132 registers; the UMOV-materialised
   // immediates stay)
-  const bool cbank = false;
+  // A DFMA takes a 32-bit immediate (the high word of the double); any other fp64
+  // coefficient is materialised by two UMOVs into a uniform register, re-issued
+  // when the 63 uniform registers run out -- on an order-4 random stencil (293
+  // coefficients) 599 UMOVs per 1172 DFMAs per plane body. From the constant
+  // bank ptxas loads two coefficients per LDCU.128 instead (176 per body).
+  // Measured on C5's 1024^3 random stencils (ST_BM_RT_PR, same box): order 3
+  // (163 coefficients) 93.0 -> 99.4 GStencil/s, order 4 (293) 54.9 -> 57.0,
+  // order 2 (51) 242 -> 233, C4's box125 (dyadic, all immediates) 124 -> 109:
+  // the constant bank pays only for large tables of non-immediate coefficients.
+  int nonimm = 0;
+  for (int i = 0; i < pat.nnz && !f32; ++i) {
+    uint64_t bits;
+    memcpy(&bits, &pat.c[i], sizeof bits);
+    nonimm += (bits & 0xffffffffull) != 0;
+  }
+  bool cbank = !f32 && nonimm >= 128;
+  if (const char* cb = getenv("STENCIL_CBANK")) cbank = atoi(cb) != 0;   // dev override
   o << (cbank ? "__constant__ " : "__device__ constexpr ") << T << " g_coef[" << pat.nnz << "] = {";
   for (int i = 0; i < pat.nnz; ++i) o << hexfloat(pat.c[i], f32) << (i + 1 < pat.nnz ? "," : "");
   o << "};\n";
@@ -423,6 +444,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   o << "  static constexpr int TMID = " << tmid << ";\n";
   o << "  static constexpr int MVX = " << (v.midvx > 0 ? v.midvx : std::max(v.vx, 1)) << ";\n";
   o << "  static constexpr bool SPLITMID = " << (v.splitmid ? "true" : "false") << ";\n";
+  o << "  static constexpr bool FULLW = " << (v.fullw ? "true" : "false") << ";\n";
   {   // k_stream_tb_rt hand-off details, off by default: measured on C2 (same box,
       // 2 runs each) elected-lane arrivals 552 -> 546 GStencil/s, warp-aligned
       // stage-1 tiles 552 -> 530, both 528 (dev overrides for A/B measurements)

@@ -88,6 +88,7 @@ struct Variant {
   bool xshift = false;        // k_stream_tb_rt: per-step ring geometry with aligned windows
   bool splitmid = false;      // k_stream_tb_rt: even/odd-split rows in the last intermediate ring
   int midvx = 0;              // k_stream_tb_rt: columns per thread of the intermediate steps (0 = vx)
+  bool fullw = false;         // k_stream_tb_rt: scalar-column stage tiles span whole ring rows (TbRtStage::FULLW)
   int tiled_mid = 0;          // k_tiled (TB): rows of the 1 x n intermediate-step register tiles (0 = scalar)
   bool flat = false;          // 2-D streaming view [ny][1][nx]: every plane is one row
   bool xm = false;            // merging (BM/CM, factor m) along x instead of y (2-D streaming view)
