@@ -268,6 +268,14 @@ __host__ __device__ constexpr int split_off(int lx, int k) {
   return lx / 2 + ((8 + (k & 1) - (lx / 2) % 16) + 32) % 16;
 }
 __host__ __device__ constexpr int split_pitch(int lx, int k) { return split_off(lx, k) + lx / 2 + 1; }
+// full-width stage tiles (FULLW, tile rows MI ring rows apart): a phase that
+// crosses from tile row cy to cy+1 continues the banks of its first part when
+// MI * SP = LX/2 (mod 16 words); solvable for odd MI
+__host__ __device__ constexpr int split_pitch_full(int lx, int so, int mi) {
+  for (int sp = so + lx / 2; sp < so + lx / 2 + 16; ++sp)
+    if (((mi * sp - lx / 2) % 16 + 16) % 16 == 0) return sp;
+  return so + lx / 2 + (16 - so % 16) % 16;
+}
 
 template <class T, int VX, int NROW>
 struct GlobalPlane {                  // global memory through the read-only path
@@ -576,7 +584,11 @@ struct TiledCfg {
   // S::TMID > 0: intermediate steps in 1 x TMID register tiles (op table S::Mid,
   // gather); the last tile of a column may read TMID - 1 rows past the buffer
   static constexpr int PAD = (TT > 1 && S::TMID > 0) ? ((S::TMID * LX * (int)sizeof(T) + 127) / 128) * 128 / (int)sizeof(T) : 0;
-  static constexpr int SMEM = (NBUF * BUF + PAD) * (int)sizeof(T) + 128;
+  // S::TFULL: the intermediate tiles span the buffer's whole rows (column 0 reads
+  // XLO elements before the first row: front pad)
+  static constexpr bool FULL = TT > 1 && S::TMID > 0 && S::TFULL;
+  static constexpr int PADF = FULL ? 128 / (int)sizeof(T) : 0;
+  static constexpr int SMEM = (NBUF * BUF + PAD + PADF) * (int)sizeof(T) + 128;
   static constexpr int THREADS = (BX / VX) * BY;
 };
 
@@ -587,9 +599,10 @@ k_tiled(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, G
   typedef typename S::T T;
   typedef TiledCfg<S, BX, BY, BZ, VX, M, CM, TT> C;
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  T* buf0 = reinterpret_cast<T*>(smem_raw);
+  T* buf0 = reinterpret_cast<T*>(smem_raw) + C::PADF;
   T* buf1 = buf0 + C::BUF;
-  unsigned long long* bar = reinterpret_cast<unsigned long long*>(smem_raw + (C::NBUF * C::BUF + C::PAD) * sizeof(T));
+  unsigned long long* bar =
+      reinterpret_cast<unsigned long long*>(smem_raw + (C::NBUF * C::BUF + C::PAD + C::PADF) * sizeof(T));
 
   const int tid = threadIdx.y * (BX / VX) + threadIdx.x;
   const int xa = (g.cx0 / C::ALN) * C::ALN;            // aligned x origin of the tile grid
@@ -640,10 +653,15 @@ k_tiled(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, G
       // 1 x MT register tiles: neighbouring lanes take neighbouring columns, so
       // every shared-memory access is a contiguous warp access, and each loaded
       // value feeds up to MT outputs of the column
-      constexpr int MT = S::TMID, NTY = (RY + MT - 1) / MT, NT = RX * NTY * RZ;
+      // C::FULL: the tiles cover every column of the buffer rows (LX), so the
+      // lanes of a 16-lane phase read consecutive words even where the phase
+      // crosses a row end (conflict-free when (MT - 1) * LX = 0 mod 16 words);
+      // the extra columns compute don't-care values the last step never reads
+      constexpr int MT = S::TMID, NTY = (RY + MT - 1) / MT;
+      constexpr int TX = C::FULL ? C::LX : RX, X1 = C::FULL ? C::XOFF : hx0, NT = TX * NTY * RZ;
       for (int t = tid; t < NT; t += C::THREADS) {
-        const int rx = t % RX, ty = (t / RX) % NTY, rz = t / (RX * NTY);
-        const int gx = xb - hx0 + rx, gy0 = yb - hy0 + ty * MT, gz = zb - hz0 + rz;
+        const int rx = t % TX, ty = (t / TX) % NTY, rz = t / (TX * NTY);
+        const int gx = xb - X1 + rx, gy0 = yb - hy0 + ty * MT, gz = zb - hz0 + rz;
         const int lb = ((gz - Z0) * C::LY + (gy0 - Y0)) * C::LX + (gx - X0);
         T acc[MT][1];
         zero_acc<T, 1, MT>(acc);
@@ -1223,12 +1241,12 @@ struct StreamTbRtCfg {
   static constexpr int MVS = S::MVX;
   static constexpr int K = XOFF - ((S::XLO + MVS - 1) / MVS) * MVS;
   // FULLW: a phase may span two tile rows, so rows must continue each other's
-  // banks (SP = LX/2 mod 16) besides the even/odd halves (SO = 8 mod 16, the
+  // banks (split_pitch_full) besides the even/odd halves (SO = 8 mod 16, the
   // phases start on even columns)
   static constexpr bool FW = S::FULLW && !S::XSHIFT && MVS == 1;
   static constexpr int SO = split_off(LX, FW ? 0 : K);
-  static constexpr int SP = !S::SPLITMID ? LX : FW ? SO + LX / 2 + (16 - SO % 16) % 16 : split_pitch(LX, K);
   static constexpr int MI = S::MI;
+  static constexpr int SP = !S::SPLITMID ? LX : FW ? split_pitch_full(LX, SO, MI) : split_pitch(LX, K);
   // slot stride: the plane plus the rows a VX x MI intermediate tile of the last
   // tile row reads past it (discarded values) -- without the gap those reads fall
   // into the next slot while the producer refills it (a benign data race that

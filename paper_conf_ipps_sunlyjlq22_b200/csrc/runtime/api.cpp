@@ -129,6 +129,10 @@ static void default_params(uint32_t oc, int ndim, int dtype, stencil_params_t* p
     // with register-tiled intermediate steps bx 64 -> 675, bx 32 -> 623; order 2:
     // 487 vs 436)
     if (ndim == 2) { p->bz = 1; p->bx = 32 * vmax; if (merge) p->merge = 4; }
+    // 2-D TB with merging: 64 x 32 tiles (round 2, with the full-width 1 x 5
+    // intermediate tiles; N2 same box: order 2 484 -> 527, order 1 642 -> 657
+    // against 64 x 16)
+    if (ndim == 2 && merge && (oc & STENCIL_OC_TB)) p->by = 8;
   } else if (fam == FAM_STREAM) {
     // wide, shallow tiles: many small CTAs keep more TMA planes in flight per SM
     // (measured on C2: 128x2 fp64 tiles reach 92% of the copy bandwidth)
@@ -370,8 +374,17 @@ static int resolve_variant(stencil_plan_s* P) {
     // (same box, TB_BM / TB): N2 order-1 8192^2 582 -> 673 / 391 -> 439, order-2
     // 423 -> 486, C2 heat 512^3 191 -> 240 / 138 -> 192 GStencil/s against one
     // point per thread; 1 x 2 is within +-4%, 1 x 8 loses
-    v.tiled_mid = 4;
-    if (const char* e = getenv("STENCIL_TILED_MID")) v.tiled_mid = std::max(0, std::min(8, atoi(e)));   // dev override
+    // Round 2: the tiles span the buffer's whole rows (TiledCfg::FULL) and are
+    // 1 x 5, so that no 16-lane phase of their loads and stores hits a bank twice
+    // where it crosses a row end ((5 - 1) * LX = 0 mod 16 words for fp64 rows of
+    // LX = 0 mod 4). ncu: the 1 x 4 tiles over the region's own columns put
+    // 12.2 M bank-conflict replays into N2 order 2's 70.3 M shared wavefronts
+    // per 2-step launch, with the L1/shared pipe 97% busy. Same box: N2 order 2
+    // (TB_BM, 64 x 32 tiles) 499 -> 527, order 1 627 -> 657, C2 heat TB_BM 192 -> 226.
+    v.tiled_mid = 5;
+    v.tiled_full = true;
+    if (const char* e = getenv("STENCIL_TILED_MID")) v.tiled_mid = std::max(0, std::min(8, atoi(e)));   // dev override (op tables encode M <= 8)
+    if (const char* e = getenv("STENCIL_TILED_FULL")) v.tiled_full = atoi(e) != 0;   // dev override
   }
   const int thr = v.threads();
   if (thr < 32 || thr > 1024)

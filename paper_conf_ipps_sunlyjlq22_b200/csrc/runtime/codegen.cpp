@@ -204,7 +204,8 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     const int lz = bz + tt * (p.zlo + p.zhi);
     const int buf = roundup(lx * ly * lz * elem, 128) / elem;
     const int pad = tt > 1 && tiled_mid > 0 ? roundup(tiled_mid * lx * elem, 128) / elem : 0;   // TiledCfg::PAD
-    return ((tt > 1 ? 2 : 1) * buf + pad) * elem + 128;
+    const int padf = tt > 1 && tiled_mid > 0 && tiled_full ? 128 / elem : 0;                      // TiledCfg::PADF
+    return ((tt > 1 ? 2 : 1) * buf + pad + padf) * elem + 128;
   }
   if (family == FAM_STREAM) {
     const int xoff = roundup(p.xlo, aln);
@@ -223,7 +224,13 @@ int Variant::smem_bytes(const Pattern& p, int elem) const {
     const int mv = midvx > 0 ? midvx : vx;
     const int k = xoff - roundup(p.xlo, mv);
     const int so = lx / 2 + ((8 + ((fullw ? 0 : k) & 1) - (lx / 2) % 16) + 32) % 16;
-    const int sp = !splitmid ? lx : fullw ? so + lx / 2 + (16 - so % 16) % 16 : so + lx / 2 + 1;
+    int sp = !splitmid ? lx : so + lx / 2 + 1;
+    if (splitmid && fullw) {                      // split_pitch_full
+      const int mi = mid_rows(p, elem);
+      sp = so + lx / 2 + (16 - so % 16) % 16;
+      for (int c = so + lx / 2; c < so + lx / 2 + 16; ++c)
+        if (((mi * c - lx / 2) % 16 + 16) % 16 == 0) { sp = c; break; }
+    }
     const int plane = roundup((std::max(lx, sp) * ly + mid_rows(p, elem) * lx + aln) * elem, 128) / elem;
     const int padf = 128 / elem;
     const int padb = roundup((mid_rows(p, elem) * lx + aln) * elem, 128) / elem;
@@ -442,6 +449,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   o << "  static constexpr int MINB = " << minb << ";\n";
   o << "  static constexpr int MIDR = " << v.mid_slots() << ";\n";
   o << "  static constexpr int TMID = " << tmid << ";\n";
+  o << "  static constexpr bool TFULL = " << (tmid > 0 && v.tiled_full ? "true" : "false") << ";\n";
   o << "  static constexpr int MVX = " << (v.midvx > 0 ? v.midvx : std::max(v.vx, 1)) << ";\n";
   o << "  static constexpr bool SPLITMID = " << (v.splitmid ? "true" : "false") << ";\n";
   o << "  static constexpr bool FULLW = " << (v.fullw ? "true" : "false") << ";\n";

@@ -28,6 +28,10 @@ CASES = {  # name: (stencil, dims, dtype, OC, params, steps)
     "tbrt_t3_fp32": ("star25", (12, 30, 72), "f32", "ST_TB_RT_PR", {"tb_steps": 3}, 4),
     "xmerge_2d": ("random2d:2:4", (40, 300), "f64", "ST_CM_RT_PR", None, 3),
     "tbrt_2d": ("random2d:1:0", (40, 300), "f64", "ST_TB_BM_RT_PR", None, 3),
+    # round 2: full-width 1 x 5 intermediate tiles of k_tiled (their x-neighbour
+    # reads run into the front pad / the neighbouring row), 2-D and fp32
+    "tiled_tb_2d": ("random2d:2:4", (70, 300), "f64", "TB_BM", None, 3),
+    "tiled_tb_fp32": ("star25", (14, 22, 72), "f32", "TB_CM", {"tb_steps": 2}, 3),
 }
 
 
