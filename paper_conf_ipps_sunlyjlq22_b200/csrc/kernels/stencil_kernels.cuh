@@ -657,26 +657,40 @@ k_tiled(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, G
       // lanes of a 16-lane phase read consecutive words even where the phase
       // crosses a row end (conflict-free when (MT - 1) * LX = 0 mod 16 words);
       // the extra columns compute don't-care values the last step never reads
-      constexpr int MT = S::TMID, NTY = (RY + MT - 1) / MT;
-      constexpr int TX = C::FULL ? C::LX : RX, X1 = C::FULL ? C::XOFF : hx0, NT = TX * NTY * RZ;
+      // S::TMVX = 2 (with FULL): MV = 2 columns per tile, 16-byte vector loads
+      // and stores -- a radius-2 row window is 3 vectors for 2 columns instead
+      // of 5 scalars for 1 (the rows start 16-byte aligned: XOFF and LX are
+      // multiples of ALN)
+      constexpr int MT = S::TMID, MV = C::FULL ? S::TMVX : 1, NTY = (RY + MT - 1) / MT;
+      constexpr int TX = C::FULL ? C::LX / MV : RX, X1 = C::FULL ? C::XOFF : hx0, NT = TX * NTY * RZ;
       for (int t = tid; t < NT; t += C::THREADS) {
         const int rx = t % TX, ty = (t / TX) % NTY, rz = t / (TX * NTY);
-        const int gx = xb - X1 + rx, gy0 = yb - hy0 + ty * MT, gz = zb - hz0 + rz;
+        const int gx = xb - X1 + rx * MV, gy0 = yb - hy0 + ty * MT, gz = zb - hz0 + rz;
         const int lb = ((gz - Z0) * C::LY + (gy0 - Y0)) * C::LX + (gx - X0);
-        T acc[MT][1];
-        zero_acc<T, 1, MT>(acc);
-        SmemPlane<T, 1, C::LX> pl[S::NZ];
+        T acc[MT][MV];
+        zero_acc<T, MV, MT>(acc);
+        SmemPlane<T, MV, C::LX> pl[S::NZ];
 #pragma unroll
         for (int zi = 0; zi < S::NZ; ++zi) pl[zi].p = src + lb + (zi - S::ZLO) * C::LY * C::LX;
-        run_gather_ops<S, typename S::Mid, 1, MT>(pl, acc);
-        const bool colok = gx >= 0 && gx < g.nx && gz >= 0 && gz < g.nz;
-        const bool colupd = gz >= g.uz0 && gz < g.uz1 && gx >= g.ux0 && gx < g.ux1;
+        run_gather_ops<S, typename S::Mid, MV, MT>(pl, acc);
+        const bool zok = gz >= 0 && gz < g.nz, zupd = gz >= g.uz0 && gz < g.uz1;
+        const bool vfast = MV > 1 && zupd && gx >= g.ux0 && gx + MV <= g.ux1;   // whole vector updated
 #pragma unroll
         for (int m = 0; m < MT; ++m) {
           const int gy = gy0 + m;
-          if (!colok || ty * MT + m >= RY || gy < 0 || gy >= g.ny) continue;
+          if (!zok || ty * MT + m >= RY || gy < 0 || gy >= g.ny) continue;
           const int li = lb + m * C::LX;
-          dst[li] = (colupd && gy >= g.uy0 && gy < g.uy1) ? acc[m][0] : src[li];
+          const bool yupd = gy >= g.uy0 && gy < g.uy1;
+          if (vfast && yupd) {
+            stg_vec<T, MV>(dst + li, acc[m]);
+            continue;
+          }
+#pragma unroll
+          for (int v = 0; v < MV; ++v) {
+            const int x = gx + v;
+            if (x < 0 || x >= g.nx) continue;
+            dst[li + v] = (zupd && yupd && x >= g.ux0 && x < g.ux1) ? acc[m][v] : src[li + v];
+          }
         }
       }
       __syncthreads();

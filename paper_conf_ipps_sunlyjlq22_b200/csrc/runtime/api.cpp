@@ -385,6 +385,14 @@ static int resolve_variant(stencil_plan_s* P) {
     v.tiled_full = true;
     if (const char* e = getenv("STENCIL_TILED_MID")) v.tiled_mid = std::max(0, std::min(8, atoi(e)));   // dev override (op tables encode M <= 8)
     if (const char* e = getenv("STENCIL_TILED_FULL")) v.tiled_full = atoi(e) != 0;   // dev override
+    // 2-column (16-byte vector) tiles where they cut the window loads or the
+    // instruction count: 3-D views and x-extent >= 3. Same box, 10 steps (TB_BM,
+    // GStencil/s, 1 column -> 2): N2 order 2 517 -> 536, order 3 253 -> 286, C2
+    // heat 217 -> 240, C5 order 2 (1024^3) 14.6 -> 22.3; the 2-D order-1 stencil
+    // (x-extent 2) loses, 647 -> 575 (56 registers: 4 CTAs per SM instead of 5)
+    v.tiled_mvx = (P->ndim == 3 || P->pat.xlo + P->pat.xhi >= 3) ? 2 : 1;
+    if (const char* e = getenv("STENCIL_TILED_MVX")) v.tiled_mvx = atoi(e) == 2 ? 2 : 1;   // dev override
+    if (!v.tiled_full || v.vx < v.tiled_mvx) v.tiled_mvx = 1;   // vector tiles need whole (aligned) rows
   }
   const int thr = v.threads();
   if (thr < 32 || thr > 1024)

@@ -429,7 +429,8 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   const int tmid = v.family == FAM_TILED && v.tt > 1 ? v.tiled_mid : 0;
   if (tmid > 0) {                      // k_tiled intermediate steps: 1 x tmid tiles, gather
     Variant vm = v;
-    vm.family = FAM_STREAM; vm.rt = false; vm.cm = false; vm.xm = false; vm.m = tmid; vm.vx = 1; vm.xshift = false;
+    vm.family = FAM_STREAM; vm.rt = false; vm.cm = false; vm.xm = false; vm.m = tmid; vm.vx = v.tiled_mvx;
+    vm.xshift = false;
     mops = encode_ops(pat, vm, pair);
   }
   if (v.family == FAM_STREAM_TB) {     // intermediate fused steps: VX x MI tiles, gather or (RT) scatter
@@ -450,6 +451,7 @@ std::string generate_source(const Pattern& pat, int dtype, const Variant& v) {
   o << "  static constexpr int MIDR = " << v.mid_slots() << ";\n";
   o << "  static constexpr int TMID = " << tmid << ";\n";
   o << "  static constexpr bool TFULL = " << (tmid > 0 && v.tiled_full ? "true" : "false") << ";\n";
+  o << "  static constexpr int TMVX = " << (tmid > 0 ? v.tiled_mvx : 1) << ";\n";
   o << "  static constexpr int MVX = " << (v.midvx > 0 ? v.midvx : std::max(v.vx, 1)) << ";\n";
   o << "  static constexpr bool SPLITMID = " << (v.splitmid ? "true" : "false") << ";\n";
   o << "  static constexpr bool FULLW = " << (v.fullw ? "true" : "false") << ";\n";

@@ -91,6 +91,7 @@ struct Variant {
   bool fullw = false;         // k_stream_tb_rt: scalar-column stage tiles span whole ring rows (TbRtStage::FULLW)
   int tiled_mid = 0;          // k_tiled (TB): rows of the 1 x n intermediate-step register tiles (0 = scalar)
   bool tiled_full = false;    // k_tiled (TB): those tiles span the buffer's whole rows (TiledCfg::FULL)
+  int tiled_mvx = 1;          // k_tiled (TB): columns of those tiles (1, or vx with tiled_full)
   bool flat = false;          // 2-D streaming view [ny][1][nx]: every plane is one row
   bool xm = false;            // merging (BM/CM, factor m) along x instead of y (2-D streaming view)
   std::string name_expr(const char* desc) const;
