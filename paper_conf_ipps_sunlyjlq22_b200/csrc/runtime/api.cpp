@@ -145,6 +145,11 @@ static void default_params(uint32_t oc, int ndim, int dtype, stencil_params_t* p
     // 64 x 32-row output tiles (8 threads x merge 4 rows), 3 planes in flight
     p->vx = vmax; p->bx = 32 * vmax; p->by = 8; p->bz = 1;
     if (merge) p->merge = 4;
+    // without merging: 64 x 16 output tiles (one row per last-stage thread), so
+    // the tile keeps its 1-row x/y halo small against its rows. Measured on C2
+    // (round 2, same box, 10 steps): ST_TB_RT_PR 303 -> 437, ST_TB_RT (no
+    // prefetching) 127 -> 210 GStencil/s against 64 x 8
+    else if (ndim == 3) p->by = 16;
     // 4 planes in flight: the stage-1 warps waited on the input ring for 23% of
     // their ncu stall samples with 3 (round 2, C2 same box: 563 -> 585 GStencil/s
     // with 4; 6: 585; 8 no longer fits one CTA per SM)
