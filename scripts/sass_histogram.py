@@ -24,13 +24,15 @@ CASES = [  # (workload, stencil, dims, dtype, OC the round-2 bench labels)
     ("C4", "box125", (512, 512, 512), "f64", "ST_CM_RT_PR"),
     ("C5", "random3d:1:0", (1024, 1024, 1024), "f64", "ST_TB_BM_RT_PR"),
     ("C5", "random3d:2:4", (1024, 1024, 1024), "f64", "ST_BM_RT_PR"),
+    ("C5", "random3d:3:8", (1024, 1024, 1024), "f64", "ST_BM_RT_PR"),
     ("C5", "random3d:4:12", (1024, 1024, 1024), "f64", "ST_BM_RT_PR"),
     ("N2", "random2d:1:0", (8192, 8192), "f64", "TB_BM"),
+    ("N2", "random2d:2:4", (8192, 8192), "f64", "TB_BM"),
     ("N2", "random2d:3:8", (8192, 8192), "f64", "ST_BM_RT_PR"),
     ("unaligned rows", "edge:asym3d", (64, 64, 67), "f64", "ST_TB_BM_RT_PR"),
 ]
 KEYS = ["UTMALDG", "UTMASTG", "UBLKCP", "LDGSTS", "SYNCS", "BAR", "LDS", "STS", "LDG", "STG", "SHFL", "DFMA",
-        "DADD", "DMUL", "FFMA", "FFMA2", "IMAD", "IADD3", "BRA", "USETMAXREG"]
+        "DADD", "DMUL", "FFMA", "FFMA2", "UMOV", "LDCU", "IMAD", "IADD3", "BRA", "USETMAXREG"]
 
 
 def main():
