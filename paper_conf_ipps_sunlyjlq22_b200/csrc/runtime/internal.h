@@ -230,6 +230,16 @@ struct stencil_plan_s {
   std::vector<cudaEvent_t> ev_pool;      // pairs: [2i] before, [2i+1] after launch i
   size_t ev_used = 0;
 
+  // CUDA graph of one stencil_run (single-domain plans): the launch sequence of
+  // the last (in, out, workspace, steps), captured at its second identical call
+  cudaGraphExec_t g_exec = nullptr;
+  cudaStream_t g_stream = nullptr;     // capture stream (the caller's may be the legacy stream)
+  const void* g_in = nullptr;
+  void* g_out = nullptr;
+  void* g_ws = nullptr;
+  int g_steps = -1, g_calls = 0;
+  uint64_t g_nlaunch = 0;              // kernels per replay (stencil_launch_count)
+
   // multi-GPU
   smart_rt::Comm* comm = nullptr;
 

@@ -419,3 +419,30 @@ def test_full_grid_elementwise(gpu, cfg, oc):
     del x
     torch.cuda.empty_cache()
     assert _relerr(got, ref) <= TOL[dtype], oc
+
+
+@pytest.mark.parametrize("oc, prm", [("base", None), ("TB_BM", None), ("ST_TB_BM_RT_PR", None)])
+def test_graph_replay(gpu, oc, prm):
+    """Round 2: stencil_run replays a CUDA graph of its launch sequence from the
+    second identical (in, out, workspace, steps) call on (api.cpp run_device).
+    Every call -- eager, captured, replayed, after a key change -- must give the
+    oracle's result, and every call must count the same kernel launches."""
+    torch = _torch()
+    acc, c = si.config_stencil("random3d:1:0")
+    dims = (20, 22, 68)
+    u0 = si.make_field(dims, 5, "f64")
+    p = sm.Plan(dims, acc, c, "f64", oc, prm)
+    x = _to_dev(u0, "f64")
+    y = torch.empty_like(x)
+    z = torch.empty_like(x)
+    refs = {s: oracle.sweep(u0, acc, c, s) for s in (3, 4)}
+    counts = []
+    for steps, out in ((3, y), (3, y), (3, y), (3, y), (4, y), (4, y), (4, y), (3, z), (3, z), (3, z), (3, y)):
+        out.fill_(float("nan"))
+        n0 = sm.launch_count()
+        p.run(x, out, steps)
+        torch.cuda.synchronize()
+        counts.append((steps, sm.launch_count() - n0))
+        assert _relerr(out.cpu().numpy(), refs[steps]) <= 1e-12, (oc, steps, len(counts))
+    for s in (3, 4):
+        assert len({n for st, n in counts if st == s}) == 1, counts
