@@ -1286,64 +1286,6 @@ struct StreamTbRtCfg {
   static constexpr int THREADS = 32 * NW;
 };
 
-// Work of one k_stream_tb_rt CTA as segments (x tile, y tile, output planes
-// [zs, ze)); every role of the CTA walks the same sequence, so the ring slots
-// and mbarrier phases simply continue from one segment to the next.
-//   chunk > 0: the CTA's (blockIdx.x, .y, .z) tile and z-chunk (one segment).
-//   chunk < 0: persistent schedule, 1-D grid of (about) one CTA per SM, used
-//              when the (x,y) columns are fewer than the CTAs (C2: 128 columns
-//              on 148 SMs): CTA b < ncols streams column b's first PA = -chunk
-//              output planes; the remaining CTAs share the columns' other
-//              planes, column-major, in equal runs. The host picks PA so that
-//              both groups finish together (api.cpp launch_sweep).
-struct TbSeg { int xb, yb, zs, ze; };
-template <int BX, int ROWS>
-struct TbSegIter {
-  int state, w, e, pa, nzc, gxn;
-  __device__ __forceinline__ TbSegIter(const Grid& g, int chunk, int xa) {
-    state = 0; w = e = 0; pa = -chunk;
-    nzc = g.cz1 - g.cz0;
-    gxn = (g.cx1 - xa + BX - 1) / BX;
-    const int ncols = gxn * ((g.cy1 - g.cy0 + ROWS - 1) / ROWS);
-    if (chunk < 0 && (int)blockIdx.x >= ncols) {
-      const long long R = (long long)ncols * max(nzc - pa, 0);
-      const long long nb = (long long)gridDim.x - ncols;
-      const long long per = (R + nb - 1) / nb, a = (long long)(blockIdx.x - ncols) * per;
-      w = (int)min(a, R);
-      e = (int)min(a + per, R);
-      state = 2;
-    }
-  }
-  __device__ __forceinline__ bool next(const Grid& g, int chunk, int xa, TbSeg& sg) {
-    if (chunk > 0) {
-      if (state) return false;
-      state = 1;
-      sg.xb = xa + blockIdx.x * BX;
-      sg.yb = g.cy0 + blockIdx.y * ROWS;
-      sg.zs = g.cz0 + blockIdx.z * chunk;
-      sg.ze = min(sg.zs + chunk, g.cz1);
-      return true;
-    }
-    if (state == 0) {                                   // phase A: column blockIdx.x
-      state = 1;
-      const int c = blockIdx.x;
-      sg.xb = xa + (c % gxn) * BX;
-      sg.yb = g.cy0 + (c / gxn) * ROWS;
-      sg.zs = g.cz0;
-      sg.ze = g.cz0 + min(pa, nzc);
-      return true;
-    }
-    if (state == 1 || w >= e) return false;             // phase B: run [w, e)
-    const int lb = nzc - pa, c = w / lb, z0 = w - c * lb, n = min(lb - z0, e - w);
-    sg.xb = xa + (c % gxn) * BX;
-    sg.yb = g.cy0 + (c / gxn) * ROWS;
-    sg.zs = g.cz0 + pa + z0;
-    sg.ze = sg.zs + n;
-    w += n;
-    return true;
-  }
-};
-
 template <class S, int BX, int BY, int VX, int M, bool CM, int NS, int TT>
 __global__ void __launch_bounds__(StreamTbRtCfg<S, BX, BY, VX, M, CM, NS, TT>::THREADS, S::MINB)
 k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__ out, Grid g, int chunk,
@@ -1369,9 +1311,13 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
   const int warp = tid >> 5;
   constexpr int AL = S::ELECT ? 1 : 32;                // arrivals per consumer warp
   const int xa = (g.cx0 / C::ALN) * C::ALN;
-  constexpr int ROWS = BY * C::TG::MY;
-  // per segment: first input plane pin0 = zs - TT*ZLO, planes each stage consumes
-  // nin = (ze - zs) + TT*(NZ - 1), box origin X0 = xb - XOFF, Y0 = yb - TT*YLO
+  const int xb = xa + blockIdx.x * BX;
+  const int yb = g.cy0 + blockIdx.y * BY * C::TG::MY;
+  const int zs = g.cz0 + blockIdx.z * chunk;
+  const int ze = min(zs + chunk, g.cz1);
+  const int pin0 = zs - TT * S::ZLO;                   // first input plane
+  const int nin = (ze - zs) + TT * (NZ - 1);           // planes each stage consumes
+  const int X0 = xb - C::XOFF, Y0 = yb - TT * S::YLO;
 
   // stage planes start defined (their unwritten corners only feed discarded outputs)
   for (int i = tid; i < C::ELEMS; i += C::THREADS) sbase[i] = T(0);
@@ -1400,50 +1346,42 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
 
   // ------------------------------------------------------------ producer
   if (warp == 0) {
-    TbSegIter<BX, ROWS> it(g, chunk, xa);
-    TbSeg sg;
-    int slot = 0, jg = 0;                                // jg: planes issued by this CTA so far
-    unsigned ph = 0;                                     // (jg / NR) & 1
     if constexpr (S::TMA) {
       if (tid == 0) {
-        while (it.next(g, chunk, xa, sg)) {
-          const int pin0 = sg.zs - TT * S::ZLO, nin = (sg.ze - sg.zs) + TT * (NZ - 1);
-          const int X0 = sg.xb - C::XOFF, Y0 = sg.yb - TT * S::YLO;
+        int slot = 0;
+        unsigned ph = 0;                                 // (j / NR) & 1
 #pragma unroll 1
-          for (int j = 0; j < nin; ++j, ++jg) {
-            if (jg >= NR) mbar_wait_sleep(&empty_in[slot], ph ^ 1u);
-            mbar_expect_tx(&full_in[slot], C::LX * C::LY * (unsigned)sizeof(T));
-            tma_load_3d(ring0 + slot * C::PLANE, &tmap, &full_in[slot], X0, Y0, pin0 + j);
-            if (++slot == NR) { slot = 0; ph ^= 1u; }
-          }
+        for (int j = 0; j < nin; ++j) {
+          if (j >= NR) mbar_wait_sleep(&empty_in[slot], ph ^ 1u);
+          mbar_expect_tx(&full_in[slot], C::LX * C::LY * (unsigned)sizeof(T));
+          tma_load_3d(ring0 + slot * C::PLANE, &tmap, &full_in[slot], X0, Y0, pin0 + j);
+          if (++slot == NR) { slot = 0; ph ^= 1u; }
         }
       }
     } else {
       // rows not TMA-aligned: the whole warp stages planes with cp.async, one
-      // commit group per plane, NS planes in flight; plane jg - (NS-1) is
+      // commit group per plane, NS planes in flight; plane j - (NS-1) is
       // published (a plain release-arrive by every lane) once cp.async.wait_group
       // says its group has landed -- the classic multistage cp.async pipeline
       // (compute-sanitizer racecheck flagged the variant that published with
       // cp.async.mbarrier.arrive.noinc; this form is clean)
-      while (it.next(g, chunk, xa, sg)) {
-        const int pin0 = sg.zs - TT * S::ZLO, nin = (sg.ze - sg.zs) + TT * (NZ - 1);
-        const int X0 = sg.xb - C::XOFF, Y0 = sg.yb - TT * S::YLO;
+      int slot = 0;
+      unsigned ph = 0;
 #pragma unroll 1
-        for (int j = 0; j < nin; ++j, ++jg) {
-          if (jg >= NR) mbar_wait_sleep(&empty_in[slot], ph ^ 1u);
-          stage_plane_cp_async<T, C::LX, C::LY, 32>(ring0 + slot * C::PLANE, in, g, X0, Y0, pin0 + j, tid);
-          cp_async_commit();
-          if (jg >= NS - 1) {
-            cp_async_wait<NS - 1>();
-            __threadfence_block();                       // landed copies ordered before the release
-            mbar_arrive(&full_in[(jg - (NS - 1)) % NR]);
-          }
-          if (++slot == NR) { slot = 0; ph ^= 1u; }
+      for (int j = 0; j < nin; ++j) {
+        if (j >= NR) mbar_wait_sleep(&empty_in[slot], ph ^ 1u);
+        stage_plane_cp_async<T, C::LX, C::LY, 32>(ring0 + slot * C::PLANE, in, g, X0, Y0, pin0 + j, tid);
+        cp_async_commit();
+        if (j >= NS - 1) {
+          cp_async_wait<NS - 1>();
+          __threadfence_block();                         // landed copies ordered before the release
+          mbar_arrive(&full_in[(j - (NS - 1)) % NR]);
         }
+        if (++slot == NR) { slot = 0; ph ^= 1u; }
       }
       cp_async_wait<0>();
       __threadfence_block();
-      for (int j = jg - (NS - 1) > 0 ? jg - (NS - 1) : 0; j < jg; ++j) mbar_arrive(&full_in[j % NR]);
+      for (int j = nin - (NS - 1) > 0 ? nin - (NS - 1) : 0; j < nin; ++j) mbar_arrive(&full_in[j % NR]);
     }
     return;
   }
@@ -1460,7 +1398,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     constexpr int MV = G::VXM;
     constexpr bool XOVER = XO_W - G::TXL + G::NTX * MV > C::LX;
     const int t = tid - 32 * W0;
-    bool act0 = t < G::NT;
+    bool act = t < G::NT;
     // tile (column cx, row cy) of thread t. S::WALIGN: the first NXM columns of
     // every tile row (a multiple of 32) are whole warps of one tile row, the
     // remaining NTX - NXM columns of all rows go to the last warp(s); otherwise
@@ -1469,30 +1407,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     constexpr int NXM = S::WALIGN == 1 ? (G::NTX / 32) * 32 : 0, NXE = G::NTXP - NXM;
     const int cx = t < NXM * G::NTY ? t % (NXM ? NXM : 1) : NXM + (t - NXM * G::NTY) % NXE;
     const int cy = t < NXM * G::NTY ? t / (NXM ? NXM : 1) : (t - NXM * G::NTY) / NXE;
-    if (cx >= G::NTX) act0 = false;                             // (WALIGN == 2 padding lanes)
-    unsigned long long* fin = s == 1 ? full_in : full_s(s - 1);
-    unsigned long long* ein = s == 1 ? empty_in : empty_s(s - 1);
-    constexpr int DIN = s == 1 ? NR : MR;
-    T acc[NZ][MI][MV];
-#pragma unroll
-    for (int q = 0; q < NZ; ++q) zero_acc<T, MV, MI>(acc[q]);
-    // NZ unrolled plane bodies (compile-time queue rotation), or one body and
-    // a register shift of the queue for large op tables (S::RTSHIFT)
-    constexpr int UNR = S::RTSHIFT ? 1 : NZ;
-    // ring slots and mbarrier phases advance incrementally across the segments
-    // (the input ring has NS + ZHI slots, generally not a power of two: j % NR
-    // and j / NR per plane cost a dozen integer instructions on every stage
-    // warp's critical path)
-    int si = 0, so = 0, sf = 0, jg = 0;                 // slots of planes j, j (own ring), j - ZHI; planes so far
-    unsigned pin = 0, pout = 0;                          // phases (jg / DIN) & 1, (jg / MR) & 1
-    TbSegIter<BX, ROWS> it(g, chunk, xa);
-    TbSeg sg;
-    while (it.next(g, chunk, xa, sg)) {
-    const int xb = sg.xb, yb = sg.yb;
-    const int pin0 = sg.zs - TT * S::ZLO, nin = (sg.ze - sg.zs) + TT * (NZ - 1);
-    const int Y0 = yb - TT * S::YLO;
-    const bool act = act0;
-    sf = (si + NR - S::ZHI % NR) % NR;                   // (stage 1) slot of plane -ZHI of this segment
+    if (cx >= G::NTX) act = false;                              // (WALIGN == 2 padding lanes)
     const int gx0 = xb - G::TXL + cx * MV;
     const int gy0 = yb - G::HY0 + cy * MI;
     const int lb_r = (gy0 - Y0) * C::LX + (gx0 - xb + XO_R);   // tile origin in the source ring
@@ -1511,6 +1426,20 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     }
     const bool xfast = gx0 >= g.ux0 && gx0 + MV <= g.ux1 && (!XOVER || gx0 - xb + XO_W + MV <= C::LX);
     const bool fast = act && xfast && allup;
+    unsigned long long* fin = s == 1 ? full_in : full_s(s - 1);
+    unsigned long long* ein = s == 1 ? empty_in : empty_s(s - 1);
+    constexpr int DIN = s == 1 ? NR : MR;
+    T acc[NZ][MI][MV];
+#pragma unroll
+    for (int q = 0; q < NZ; ++q) zero_acc<T, MV, MI>(acc[q]);
+    // NZ unrolled plane bodies (compile-time queue rotation), or one body and
+    // a register shift of the queue for large op tables (S::RTSHIFT)
+    constexpr int UNR = S::RTSHIFT ? 1 : NZ;
+    // ring slots and mbarrier phases advance incrementally (the input ring has
+    // NS + ZHI slots, generally not a power of two: j % NR and j / NR per plane
+    // cost a dozen integer instructions on every stage warp's critical path)
+    int si = 0, so = 0, sf = (NR - S::ZHI % NR) % NR;   // slots of planes j, j (own ring), j - ZHI
+    unsigned pin = 0, pout = 0;                          // phases (j / DIN) & 1, (j / MR) & 1
 #pragma unroll 1
     for (int jb = 0; jb < nin; jb += UNR) {
       static_for<0, UNR>([&](auto ic) {
@@ -1526,7 +1455,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         }
         if (s > 1) warp_arrive<S::ELECT>(&ein[si]);      // input slot read (stage 1: below)
         T* dst = mid + (MR * (s - 1) + so) * C::PLANE;
-        if (jg >= MR) mbar_wait_sleep(&empty_s(s)[so], pout ^ 1u);
+        if (j >= MR) mbar_wait_sleep(&empty_s(s)[so], pout ^ 1u);
         const int zo = pin0 + j - s * S::ZHI;            // plane completed now
         // stage 1: input plane zo (= index j - ZHI) is still in the ring
         const T* fr = ring0 + sf * C::PLANE + lb_r;
@@ -1560,9 +1489,7 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
                 const int gx = gx0 + v;
                 if (gx < 0 || gx >= g.nx || gx - xb + XO_W >= C::LX) continue;
                 const bool upd = rowupd && gx >= g.ux0 && gx < g.ux1;
-                // (stage 1, j < ZHI: the frame plane precedes the segment; the value is
-                // a don't-care, and its slot may be refilling)
-                const T val = upd ? res[m][v] : s == 1 ? (j >= S::ZHI ? fr[m * C::LX + v] : T(0)) : __ldg(frame + gx);
+                const T val = upd ? res[m][v] : (s == 1 ? fr[m * C::LX + v] : __ldg(frame + gx));
                 if constexpr (SPL) dst[split_idx<C::SP, C::SO>(lrow + m, lcol + v)] = val;
                 else d[v] = val;
               }
@@ -1575,17 +1502,8 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
         if (++si == DIN) { si = 0; pin ^= 1u; }
         if (++so == MR) { so = 0; pout ^= 1u; }
         if (++sf == NR) sf = 0;
-        ++jg;
       });
     }
-    if (s == 1) {                                        // release the segment's last ZHI frame planes
-#pragma unroll 1
-      for (int q = 0; q < S::ZHI; ++q) {
-        warp_arrive<S::ELECT>(&ein[sf]);
-        if (++sf == NR) sf = 0;
-      }
-    }
-    }   // segments
   });
   if (done || warp < C::WL || warp >= C::WL + C::WF) return;   // (idle padding warps)
 
@@ -1597,46 +1515,39 @@ k_stream_tb_rt(const typename S::T* __restrict__ in, typename S::T* __restrict__
     const int tx = q % TG::TPX, ty = q / TG::TPX;
     const int row0 = TT * S::YLO + TG::row(ty);
     const int col0 = C::xoff(TT - 1) + tx * TG::XSTEP - S::XSH;   // window start in the last ring
+    const int x0 = xb + tx * TG::XSTEP;
+    const int y0 = yb + TG::row(ty);
+    const TileStore<T, VX, M, CM, BY, S::SY, S::SZ, TG::XS> ts(out, g, y0, x0);
     unsigned long long* fin = full_s(TT - 1);
     unsigned long long* ein = empty_s(TT - 1);
     T acc[NZ][M][VX];
 #pragma unroll
     for (int u = 0; u < NZ; ++u) zero_acc<T, VX, M>(acc[u]);
     constexpr int UNR = S::RTSHIFT ? 1 : NZ;
-    int si = 0;                                          // slot of plane jg in the last ring
-    unsigned ph = 0;                                     // (jg / MR) & 1
-    TbSegIter<BX, ROWS> it(g, chunk, xa);
-    TbSeg sg;
-    while (it.next(g, chunk, xa, sg)) {
-      const int pin0 = sg.zs - TT * S::ZLO, nin = (sg.ze - sg.zs) + TT * (NZ - 1), zs = sg.zs;
-      const int x0 = sg.xb + tx * TG::XSTEP;
-      const int y0 = sg.yb + TG::row(ty);
-      const TileStore<T, VX, M, CM, BY, S::SY, S::SZ, TG::XS> ts(out, g, y0, x0);
 #pragma unroll 1
-      for (int jb = 0; jb < nin; jb += UNR) {
-        static_for<0, UNR>([&](auto ic) {
-          constexpr int U = S::RTSHIFT ? NZ - 1 : decltype(ic)::value;
-          const int j = jb + decltype(ic)::value;
-          if (j >= nin) return;
-          mbar_wait_sleep(&fin[si], ph);
-          if constexpr (!S::RTSHIFT) zero_acc<T, VX, M>(acc[U]);
-          if (act) {
-            const T* pm = mid + (MR * (TT - 2) + si) * C::PLANE;
-            if constexpr (S::SPLITMID) {
-              SplitPlane<T, C::SP, C::SO> pl{pm + row0 * C::SP + (col0 >> 1)};
-              run_scatter<S, VX, M, U>(pl, acc);
-            } else {
-              SmemPlane<T, VX, C::LX> pl{pm + row0 * C::LX + col0};
-              run_scatter<S, VX, M, U>(pl, acc);
-            }
+    for (int jb = 0; jb < nin; jb += UNR) {
+      static_for<0, UNR>([&](auto ic) {
+        constexpr int U = S::RTSHIFT ? NZ - 1 : decltype(ic)::value;
+        const int j = jb + decltype(ic)::value;
+        if (j >= nin) return;
+        const int si = j % MR;
+        mbar_wait_sleep(&fin[si], (unsigned)((j / MR) & 1));
+        if constexpr (!S::RTSHIFT) zero_acc<T, VX, M>(acc[U]);
+        if (act) {
+          const T* pm = mid + (MR * (TT - 2) + si) * C::PLANE;
+          if constexpr (S::SPLITMID) {
+            SplitPlane<T, C::SP, C::SO> pl{pm + row0 * C::SP + (col0 >> 1)};
+            run_scatter<S, VX, M, U>(pl, acc);
+          } else {
+            SmemPlane<T, VX, C::LX> pl{pm + row0 * C::LX + col0};
+            run_scatter<S, VX, M, U>(pl, acc);
           }
-          warp_arrive<S::ELECT>(&ein[si]);
-          const int z = pin0 + j - TT * S::ZHI;
-          if (act && z >= zs) ts.store(z, acc[(U + 1) % NZ], g, out);
-          if constexpr (S::RTSHIFT) shift_queue<T, NZ, M, VX>(acc);
-          if (++si == MR) { si = 0; ph ^= 1u; }
-        });
-      }
+        }
+        warp_arrive<S::ELECT>(&ein[si]);
+        const int z = pin0 + j - TT * S::ZHI;
+        if (act && z >= zs) ts.store(z, acc[(U + 1) % NZ], g, out);
+        if constexpr (S::RTSHIFT) shift_queue<T, NZ, M, VX>(acc);
+      });
     }
   }
 }

@@ -595,33 +595,6 @@ static int launch_sweep(stencil_plan_s* P, const Variant& v, const Kernel& k, co
     } else {
       chunk = auto_chunk(P, v, k, (int)(bx * by), v.smem_bytes(P->pat, elem), czlen, (long long)gx * gy);
       gz = (czlen + chunk - 1) / chunk;
-      // k_stream_tb_rt with fewer (x,y) columns than resident CTAs (C2: 128 on
-      // 148 SMs) can run a persistent 1-D grid (TbSegIter, stencil_kernels.cuh)
-      // instead of z-chunks: chunks of 64 planes cost C2 4 fill planes each (6%)
-      // plus a 6.9-wave tail; persistent, CTA b < ncols streams PA planes of
-      // column b and the other CTAs share the rest, PA = ncols (n + F) / nCTA
-      // making both groups finish together (F = TT (NZ - 1) fill planes per
-      // segment). Measured on C2 (same box, twice): 563 vs 575 GStencil/s with
-      // the z-chunks -- the CTAs sharing the column tails no longer stream in
-      // step with their x/y neighbours, so their halo rows miss L2 -- so it is
-      // off by default. STENCIL_TBRT_PERSIST: 1 on, 2 also for short columns
-      // (the parity tests force it to exercise CTAs with many segments).
-      if (v.family == FAM_STREAM_TB && v.rt && v.chunk <= 0) {
-        const char* pe = getenv("STENCIL_TBRT_PERSIST");
-        const int persist = pe ? atoi(pe) : 0;
-        int nsm = 0, dev = 0, occ = 0;
-        if (persist && cudaGetDevice(&dev) == cudaSuccess &&
-            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess &&
-            d->occupancy(&occ, k.fn, (int)bx, (size_t)v.smem_bytes(P->pat, elem)) == CUDA_SUCCESS && occ > 0) {
-          const long long ncta = (long long)nsm * occ, ncols = (long long)gx * gy;
-          const long long f = (long long)v.tt * (P->pat.zlo + P->pat.zhi);
-          const long long pa = (ncols * (czlen + f) + ncta - 1) / ncta;
-          if (ncols < ncta && pa < czlen && (pa >= 4 * f || persist == 2)) {
-            chunk = -(int)pa;
-            gx = (unsigned)ncta; gy = 1; gz = 1;
-          }
-        }
-      }
       args[3] = (void*)&chunk;
       args[4] = tm ? (void*)tm : (void*)&dummy;
       nargs = 5;
@@ -1115,13 +1088,13 @@ void free_host_path_buffers(stencil_plan_s* P) {
 // (module loads, tensor maps), the second is captured on the plan's own stream
 // and launched, later ones only launch the graph. Small grids are launch-bound
 // (C1, 256^2: 12 launches of a few us each per run). Not used with kernel timing
-// (per-launch events), slabs (exchanges on other streams) or STENCIL_GRAPHS=0.
+// (per-launch events) or slabs (exchanges on other streams); opt-in (below).
+// Off by default: measured on C1 (256^2, 10 steps, same box, twice each) the
+// end-to-end step took 0.121-0.139 ms with graph replay against 0.107-0.111 ms
+// with direct launches. STENCIL_GRAPHS=1 turns it on.
 static bool graphs_enabled() {
-  static const bool on = [] {
-    const char* e = getenv("STENCIL_GRAPHS");
-    return !e || atoi(e) != 0;
-  }();
-  return on;
+  const char* e = getenv("STENCIL_GRAPHS");
+  return e && atoi(e) != 0;
 }
 
 static void drop_graph(stencil_plan_s* P) {

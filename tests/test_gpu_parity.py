@@ -422,12 +422,13 @@ def test_full_grid_elementwise(gpu, cfg, oc):
 
 
 @pytest.mark.parametrize("oc, prm", [("base", None), ("TB_BM", None), ("ST_TB_BM_RT_PR", None)])
-def test_graph_replay(gpu, oc, prm):
+def test_graph_replay(gpu, monkeypatch, oc, prm):
     """Round 2: stencil_run replays a CUDA graph of its launch sequence from the
     second identical (in, out, workspace, steps) call on (api.cpp run_device).
     Every call -- eager, captured, replayed, after a key change -- must give the
     oracle's result, and every call must count the same kernel launches."""
     torch = _torch()
+    monkeypatch.setenv("STENCIL_GRAPHS", "1")
     acc, c = si.config_stencil("random3d:1:0")
     dims = (20, 22, 68)
     u0 = si.make_field(dims, 5, "f64")
@@ -446,27 +447,3 @@ def test_graph_replay(gpu, oc, prm):
         assert _relerr(out.cpu().numpy(), refs[steps]) <= 1e-12, (oc, steps, len(counts))
     for s in (3, 4):
         assert len({n for st, n in counts if st == s}) == 1, counts
-
-
-@pytest.mark.parametrize("name, dims, dtype, oc", [
-    ("heat3d", (40, 36, 140), "f64", "ST_TB_BM_RT_PR"),
-    ("random3d:1:0", (37, 30, 136), "f64", "ST_TB_CM_RT"),
-    ("edge:asym3d", (33, 41, 67), "f64", "ST_TB_BM_RT_PR"),
-    ("star25", (30, 28, 72), "f32", "ST_TB_RT_PR"),
-])
-def test_tb_rt_persistent_segments(gpu, monkeypatch, name, dims, dtype, oc):
-    """Round 2: k_stream_tb_rt's persistent schedule (TbSegIter) -- CTAs that
-    stream several column segments in a row, ring slots and mbarrier phases
-    carried across them -- forced on short columns (STENCIL_TBRT_PERSIST=2),
-    10 steps, against the oracle and bitwise against the z-chunk schedule."""
-    torch = _torch()
-    acc, c = si.config_stencil(name)
-    u0 = si.make_field(dims, 11, dtype)
-    ref = oracle.sweep(u0, acc, c, 10, dtype=dtype)
-    outs = {}
-    for mode in ("0", "2"):
-        monkeypatch.setenv("STENCIL_TBRT_PERSIST", mode)
-        p = sm.Plan(dims, acc, c, dtype, oc)
-        outs[mode] = _run(p, u0, dtype, 10)
-    assert _relerr(outs["2"], ref) <= TOL[dtype]
-    assert np.array_equal(outs["0"], outs["2"])
