@@ -213,3 +213,38 @@ def test_2d_streaming_merge_along_x(dtype):
         assert bm["params"]["merge"] == 2 and base["params"]["merge"] == 1
         if suffix != "_TB_RT":
             assert bm["threads"] * bm["params"]["vx"] * 2 == bm["params"]["bx"]
+
+
+def _sass_counts(cache_dir, opcodes):
+    import glob
+    import subprocess
+    n = {op: 0 for op in opcodes}
+    for f in glob.glob(os.path.join(cache_dir, "*.cubin")):
+        sass = subprocess.run(["cuobjdump", "-sass", f], capture_output=True, text=True).stdout
+        for line in sass.splitlines():
+            m = re.match(r"\s*/\*[0-9a-f]+\*/\s+(?:@!?U?P\w+\s+)?([A-Z][A-Z0-9_]*)", line)
+            if m and m.group(1) in n:
+                n[m.group(1)] += 1
+    return n
+
+
+def test_coefficient_operands_choice(tmp_path, monkeypatch):
+    """Round 2: fp64 coefficients that are not DFMA
+    immediates come from the constant bank (LDCU) once the stencil has >= 128 of
+    them -- the order-4 Algorithm-1 stencil (293, normalised random values) --
+    instead of UMOV pairs; dyadic coefficients (box125) stay immediates. Checked
+    in the NVRTC cubins' SASS (host only)."""
+    import shutil
+    if not shutil.which("cuobjdump"):
+        pytest.skip("cuobjdump not available")
+    oc = sm.oc_from_name("ST_BM_RT_PR")
+    counts = {}
+    for name in ("random3d:4:12", "box125"):
+        d = tmp_path / name.replace(":", "_")
+        monkeypatch.setenv("STENCIL_CACHE_DIR", str(d))
+        acc, c = si.config_stencil(name)
+        _plan((41, 43, 74), acc, c, "f64", oc)     # dims unique to this test: a fresh NVRTC compile
+        counts[name] = _sass_counts(str(d), ("DFMA", "UMOV", "LDCU"))
+    r4, box = counts["random3d:4:12"], counts["box125"]
+    assert r4["DFMA"] > 1000 and r4["LDCU"] >= 100 and r4["UMOV"] < r4["DFMA"] // 20, r4
+    assert box["DFMA"] >= 125 and box["LDCU"] < 40, box
