@@ -447,3 +447,27 @@ def test_graph_replay(gpu, monkeypatch, oc, prm):
         assert _relerr(out.cpu().numpy(), refs[steps]) <= 1e-12, (oc, steps, len(counts))
     for s in (3, 4):
         assert len({n for st, n in counts if st == s}) == 1, counts
+
+
+@pytest.mark.parametrize("stencil, oc", [("random2d:1:0", "TB_BM"), ("random2d:2:4", "TB_BM"),
+                                         ("random2d:3:8", "TB_BM"), ("random2d:2:4", "TB_CM")])
+def test_full_grid_n2_tiled_tb(gpu, stencil, oc):
+    """Round 2: N2's whole 8192^2 fp64 grid after its 10 steps, element by element
+    against the oracle, through the round-2 k_tiled TB path the bench labels for
+    orders 1-2 (full-width 1 x 5 intermediate tiles, 2-column tiles for x-extent
+    >= 3, 64 x 32 tiles) -- default settings, as the bench times them."""
+    torch = _torch()
+    C = si.CONFIGS["N2"]
+    acc, c = si.config_stencil(stencil)
+    dims, dtype, steps = C["dims"], C["dtype"], C["steps"]
+    x = torch.empty(dims, dtype=torch.float64, device="cuda")
+    sm.fill_field(x, C["seed"])
+    y = torch.empty_like(x)
+    sm.Plan(dims, acc, c, dtype, sm.oc_from_name(oc)).run(x, y, steps)
+    torch.cuda.synchronize()
+    got = y.cpu().numpy()
+    del y
+    ref = oracle.sweep(x.cpu().numpy(), acc, c, steps, dtype=dtype)
+    del x
+    torch.cuda.empty_cache()
+    assert _relerr(got, ref) <= TOL[dtype], (stencil, oc)
