@@ -350,6 +350,13 @@ static int resolve_variant(stencil_plan_s* P) {
       const int l0 = count_window_loads(P->pat, elem, v), l1 = count_window_loads(P->pat, elem, vs);
       v.xshift = l1 <= 0.85 * l0;
     }
+    // 8-row block-merged last stage on a radius-1 in-plane pattern (the setting
+    // stencil_plan_create picks for C2-like stencils): measured with the rounded
+    // geometry; the aligned windows would win on load counts but took C2 from 615
+    // to 434 GStencil/s (they also rule out the scalar-column stage tiles)
+    if (v.m == 8 && !v.cm && !v.xm && elem == 8 && P->pat.xlo <= 1 && P->pat.xhi <= 1 && P->pat.ylo <= 1 &&
+        P->pat.yhi <= 1)
+      v.xshift = false;
     if (const char* nx = getenv("STENCIL_XSHIFT")) v.xshift = tma_ok && atoi(nx) != 0;   // dev override
     // even/odd-split last intermediate ring (fp64, 16-byte vectors of 2, rounded geometry)
     v.splitmid = elem == 8 && v.vx == 2 && !v.xshift;
@@ -366,8 +373,19 @@ static int resolve_variant(stencil_plan_s* P) {
     }
     if (const char* mv = getenv("STENCIL_MID_VX"))   // dev override: intermediate-step columns per thread
       if (!v.xshift) v.midvx = std::max(0, std::min(v.vx, atoi(mv)));
-    // scalar-column stage tiles over whole ring rows (TbRtStage::FULLW)
+    // scalar-column stage tiles over whole ring rows (TbRtStage::FULLW); with
+    // 8-row last-stage tiles (merge 8, see stencil_plan_create) they come with
+    // 1 x 5 stage tiles (conflict-free: (5 - 1) * LX = 0 mod 16 words) and
+    // 3-slot stage rings. C2, same box, 10 steps (GStencil/s): the round-2
+    // default (merge 4, 1 x 4 tiles, 2 slots) 590; merge 8 + these 603 (2
+    // slots) / 615 (3 slots); merge 8 alone 579
     v.fullw = false;
+    v.mid_rows_set = v.mid_slots_set = 0;
+    if (v.midvx == 1 && !v.xshift && v.m == 8 && !v.cm && !v.xm) {
+      v.fullw = true;
+      v.mid_rows_set = 5;
+      v.mid_slots_set = 3;
+    }
     if (const char* fw = getenv("STENCIL_FULLW")) v.fullw = atoi(fw) != 0;   // dev override
     if (v.midvx != 1 || v.xshift) v.fullw = false;
     if (v.fullw && v.tbrt_threads(P->pat, elem) > 1024) v.fullw = false;
@@ -1251,6 +1269,14 @@ int stencil_plan_create(stencil_plan_t* plan, int ndim, const int64_t* dims, int
       P->params.bx /= 2;
     }
   }
+  // TB-RT with block merging on a radius-1 in-plane star (C2's heat; the
+  // scalar-column stage tiles of resolve_variant): 8-row last-stage tiles, 64 x
+  // 32 outputs per CTA as before but 4 last-stage warps instead of 8 and 2.25
+  // instead of 2.5 shared loads per output (round 2)
+  const bool user_m = params && params->merge;
+  bool try_m8 = !user_by && !user_m && ndim == 3 && family_of(oc, P->params.smem) == FAM_STREAM_TB &&
+                (oc & STENCIL_OC_RT) && (oc & STENCIL_OC_BM) && dtype == STENCIL_F64 && P->params.by == 8 &&
+                P->params.merge == 4;
   std::string first_err;   // the reason at the requested (or default) setting
   for (int attempt = 0;; ++attempt) {
     const int rc = resolve_variant(P.get());
@@ -1267,6 +1293,18 @@ int stencil_plan_create(stencil_plan_t* plan, int ndim, const int64_t* dims, int
     if (!give_up) continue;
     if (rc == STENCIL_E_OC_INFEASIBLE) SM_FAIL(rc, "%s (no smaller default tile fits either)", first_err.c_str());
     if (rc != STENCIL_OK) return rc;
+    if (try_m8) {
+      try_m8 = false;
+      const char* nm = getenv("STENCIL_NO_M8");   // dev override (A/B against the round-1 setting)
+      if (P->var.midvx == 1 && !P->var.xshift && !(nm && atoi(nm))) {
+        const stencil_params_t keep = P->params;
+        P->params.by = 4;
+        P->params.merge = 8;
+        if (resolve_variant(P.get()) == STENCIL_OK && P->var.fullw) break;
+        P->params = keep;                                 // fall back to the measured round-1 setting
+        if (resolve_variant(P.get()) != STENCIL_OK) return STENCIL_E_OC_INFEASIBLE;
+      }
+    }
     break;
   }
   clear_error();

@@ -139,13 +139,14 @@ int Variant::mid_rows(const Pattern& p, int elem) const {
   if (flat) return 1;          // 2-D streaming view: a plane is one row, taller tiles only waste lanes
   if (family == FAM_STREAM_TB && rt)
     if (const char* e = getenv("STENCIL_MID_ROWS")) return atoi(e);   // dev override
+  if (mid_rows_set > 0) return mid_rows_set;
   return midvx == 1 ? 4 : 2;   // scalar-column intermediate tiles: 1 x 4
 }
 
 // Slots of each intermediate-stage ring of k_stream_tb_rt (S::MIDR).
 int Variant::mid_slots() const {
   if (const char* e = getenv("STENCIL_MIDR")) return std::max(2, atoi(e));   // dev override
-  return 2;
+  return mid_slots_set > 0 ? mid_slots_set : 2;
 }
 
 // Mirrors StreamTbRtCfg::THREADS of stencil_kernels.cuh: one producer warp,

@@ -89,6 +89,8 @@ struct Variant {
   bool splitmid = false;      // k_stream_tb_rt: even/odd-split rows in the last intermediate ring
   int midvx = 0;              // k_stream_tb_rt: columns per thread of the intermediate steps (0 = vx)
   bool fullw = false;         // k_stream_tb_rt: scalar-column stage tiles span whole ring rows (TbRtStage::FULLW)
+  int mid_rows_set = 0;       // k_stream_tb_rt: rows of the intermediate tiles when > 0 (else mid_rows' rule)
+  int mid_slots_set = 0;      // k_stream_tb_rt: slots of each stage ring when > 0 (else 2)
   int tiled_mid = 0;          // k_tiled (TB): rows of the 1 x n intermediate-step register tiles (0 = scalar)
   bool tiled_full = false;    // k_tiled (TB): those tiles span the buffer's whole rows (TiledCfg::FULL)
   int tiled_mvx = 1;          // k_tiled (TB): columns of those tiles (1, or vx with tiled_full)
