@@ -248,3 +248,24 @@ def test_coefficient_operands_choice(tmp_path, monkeypatch):
     r4, box = counts["random3d:4:12"], counts["box125"]
     assert r4["DFMA"] > 1000 and r4["LDCU"] >= 100 and r4["UMOV"] < r4["DFMA"] // 20, r4
     assert box["DFMA"] >= 125 and box["LDCU"] < 40, box
+
+
+def test_tbrt_eight_row_setting_choice():
+    """Round 2 (DESIGN.md §6.1 (4)): block-merged TB-RT on an fp64 radius-1
+    in-plane star with default parameters takes 8-row last-stage tiles (by 4 x
+    merge 8, 64 x 32 outputs) with full-width 1 x 5 stage tiles: 20 warps. An
+    explicit setting is kept; cyclic merging, the 3x3-plane order-1 Algorithm-1
+    stencil (aligned-window geometry) and fp32 keep the 64 x 32 = 8 x merge-4 tile."""
+    oc = sm.oc_from_name("ST_TB_BM_RT_PR")
+    acc, c = si.config_stencil("heat3d")
+    p = _plan((512, 512, 512), acc, c, "f64", oc)
+    assert (p.info["params"]["by"], p.info["params"]["merge"], p.info["threads"]) == (4, 8, 640)
+    assert not p.info["xshift"]
+    q = _plan((512, 512, 512), acc, c, "f64", oc, {"bx": 64, "by": 8, "vx": 2, "merge": 4, "tb_steps": 2, "pr_stages": 4})
+    assert (q.info["params"]["by"], q.info["params"]["merge"], q.info["threads"]) == (8, 4, 896)
+    r = _plan((512, 512, 512), acc, c, "f64", oc, dict(p.info["params"]))   # the label's reported setting
+    assert r.info["threads"] == 640 and not r.info["xshift"]
+    assert _plan((512, 512, 512), acc, c, "f64", sm.oc_from_name("ST_TB_CM_RT_PR")).info["params"]["merge"] == 4
+    assert _plan((512, 512, 512), acc, c, "f32", oc).info["params"]["merge"] == 4
+    acc1, c1 = si.config_stencil("random3d:1:0")
+    assert _plan((256, 256, 256), acc1, c1, "f64", oc).info["params"]["merge"] == 4
