@@ -482,22 +482,32 @@ def run_impl(args):
         return p
 
     # every rank owns dims[0] planes of a global grid of depth world*dims[0]
-    # (weak scaling); slab buffers carry G ghost planes on each side. One
-    # input/output pair (and one workspace) serves every stencil of the step.
-    probe = make_plan(items[0]["acc"], items[0]["c"], 0)
-    G = probe.ghost
-    shape = probe.array_shape
+    # (weak scaling); slab buffers carry G ghost planes on each side, G = the
+    # stencil's own depth (4 x order), so in slab mode every stencil of a
+    # multi-stencil workload (C5) gets its own input/output/workspace; otherwise
+    # one pair (and one workspace) serves every stencil of the step.
     gdims = (dims[0] * world,) + dims[1:] if len(dims) == 3 else dims
-    x = torch.zeros(shape, dtype=tdt, device=dev)
-    if len(dims) == 3:
-        z0 = dims[0] * rank
-        a, b = max(0, z0 - G), min(gdims[0], z0 + dims[0] + G)
-        sm.fill_field(x[a - (z0 - G):b - (z0 - G)], C["seed"], 0, origin=(a, 0, 0), global_dims=gdims)
-    else:
-        sm.fill_field(x, C["seed"], 0)
-    y = torch.empty_like(x)
-    ws = torch.empty(probe.workspace_bytes() // elem, dtype=tdt, device=dev)
-    del probe
+
+    def alloc_bufs(it):
+        probe = make_plan(it["acc"], it["c"], 0)
+        G = probe.ghost
+        xb = torch.zeros(probe.array_shape, dtype=tdt, device=dev)
+        if len(dims) == 3:
+            z0 = dims[0] * rank
+            a, b = max(0, z0 - G), min(gdims[0], z0 + dims[0] + G)
+            sm.fill_field(xb[a - (z0 - G):b - (z0 - G)], C["seed"], 0, origin=(a, 0, 0), global_dims=gdims)
+        else:
+            sm.fill_field(xb, C["seed"], 0)
+        bufs = (xb, torch.empty_like(xb), torch.empty(probe.workspace_bytes() // elem, dtype=tdt, device=dev), G)
+        del probe
+        return bufs
+
+    shared = None
+    for it in items:
+        if slab or shared is None:
+            shared = alloc_bufs(it)
+        it["x"], it["y"], it["ws"], it["G"] = shared
+    x, y, ws, G = items[0]["x"], items[0]["y"], items[0]["ws"], max(it["G"] for it in items)
     stream = torch.cuda.current_stream()
 
     # ---- 1. label pass per stencil: every OC of the family, seeded settings (a8)
@@ -507,6 +517,7 @@ def run_impl(args):
         ocs = [sm.oc_from_name(args.oc)]
     t_sw = time.time()
     for it in items:
+        x, y, ws = it["x"], it["y"], it["ws"]
         base_plan = make_plan(it["acc"], it["c"], 0)
         base_plan.use_workspace(ws)
         info0 = base_plan.info
@@ -603,7 +614,7 @@ def run_impl(args):
 
     def step():
         for it in items:
-            it["plan"].run(x, y, steps)
+            it["plan"].run(it["x"], it["y"], steps)
 
     # ---- 2. warm-up + timed steps (one step = every stencil of the workload)
     for _ in range(args.warmup):
@@ -621,7 +632,7 @@ def run_impl(args):
     # grids that fit the 126 MB L2 (C1: 0.5 MB) would be timed from L2: flush it
     # between the timed steps by writing a 256 MB buffer, outside the per-step
     # CUDA-event pairs (the time is their sum); larger grids stream through L2
-    grid_bytes = x.numel() * x.element_size()
+    grid_bytes = max(it["x"].numel() for it in items) * elem
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev) if 2 * grid_bytes < L2_BYTES else None
     with ClockSampler(local) as clk:
         if flush is None:
@@ -677,28 +688,36 @@ def run_impl(args):
         # (which stages into its own device buffers) does not apply
         e2e = {"value": None, "unsupported": "stencil_run_host does not run P2P-registered slab plans"}
     elif not args.no_e2e:
-        hin = torch.empty(tuple(x.shape), dtype=tdt, pin_memory=True)
-        hin.copy_(x.cpu())
+        # pinned host buffers of the largest stencil's array; each stencil runs
+        # on a view of its own (slab) shape
+        big = max(items, key=lambda it: it["x"].numel())["x"]
+        hin = torch.empty(tuple(big.shape), dtype=tdt, pin_memory=True)
+        hin.copy_(big.cpu())
         hout = torch.empty_like(hin).pin_memory()
         for it in items:
-            it["plan"].run_host(hin, hout, steps)   # warm (allocates the plan's device buffers)
+            n = it["x"].numel()
+            it["hin"] = hin.view(-1)[:n].view(tuple(it["x"].shape))
+            it["hout"] = hout.view(-1)[:n].view(tuple(it["x"].shape))
+            it["plan"].run_host(it["hin"], it["hout"], steps)   # warm (allocates the plan's device buffers)
         n_e2e = max(1, min(3, args.steps))
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         for _ in range(n_e2e):
             for it in items:
-                it["plan"].run_host(hin, hout, steps)
+                it["plan"].run_host(it["hin"], it["hout"], steps)
         torch.cuda.synchronize()
         e2e_ms = (time.perf_counter() - t0) * 1e3 / n_e2e
         if world > 1:
             t = torch.tensor([e2e_ms], device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e2e_ms = float(t.item())
-        nbytes = x.numel() * elem * len(items)
+        nbytes = sum(it["x"].numel() for it in items) * elem
         e2e = {"value": round(pts_all * steps / (e2e_ms * 1e-3) / 1e9, 3), "unit": "GStencil/s",
                "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes, "ms_per_step": round(e2e_ms, 3),
                "host_chunks": [it["plan"].info["host_chunks"] for it in items],
-               "pcie_gbs": _pcie_probe(hin, hout, x, y)}
+               "pcie_gbs": _pcie_probe(items[0]["hin"], items[0]["hout"], items[0]["x"], items[0]["y"])}
+        for it in items:
+            it.pop("hin", None), it.pop("hout", None)
         del hin, hout
 
     # ---- 5. CPU oracle beside it (rank 0, N = 1)
@@ -759,6 +778,14 @@ def run_impl(args):
 
 
 def main():
+    # stdout carries exactly one JSON line: the image sets NCCL_DEBUG=VERSION,
+    # whose banner NCCL prints to stdout at the first communicator (seen on the
+    # --slab runs); WARN keeps warnings and drops the banner, and any other log
+    # NCCL writes goes to stderr
+    if os.environ.get("NCCL_DEBUG", "").upper() == "VERSION":
+        os.environ["NCCL_DEBUG"] = "WARN"
+    if os.environ.get("NCCL_DEBUG") and not os.environ.get("NCCL_DEBUG_FILE"):
+        os.environ["NCCL_DEBUG_FILE"] = "/dev/stderr"
     ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
