@@ -1202,12 +1202,13 @@ struct TbRtStage {
   // warp access instead of 16-byte vectors with half-used neighbours)
   static constexpr int VXM = S::MVX;
   // S::FULLW (scalar columns, rounded geometry): the stage's tiles span every
-  // column of the ring rows (pitch LXF, the TMA box width), so thread t reads
-  // ring word t + const for each window element and no 16-lane phase of a load
-  // can put two tile rows on the same banks (row-straddling phases of 66-column
-  // tile rows in a 68-element pitch replayed up to 2 wavefronts each). The
-  // extra columns are computed from don't-care neighbours and never feed a
-  // valid output.
+  // column of the ring rows (pitch LXF, the TMA box width). A 16-lane phase
+  // that crosses from tile row cy to cy+1 then jumps (MI - 1) * LXF words, so
+  // with (MI - 1) * LXF = 0 mod 16 (C2: MI = 5, LXF = 68) no load phase puts
+  // two tile rows on the same banks (row-straddling phases of 66-column tile
+  // rows in a 68-element pitch replayed up to 2 wavefronts each). The extra
+  // columns are computed from don't-care neighbours and never feed a valid
+  // output.
   static constexpr bool FULLW = S::FULLW && !S::XSHIFT && VXM == 1;
   static constexpr int ALNF = (16 / (int)sizeof(typename S::T)) > VX ? (16 / (int)sizeof(typename S::T)) : VX;
   static constexpr int XOFFF = ((TT * S::XLO + ALNF - 1) / ALNF) * ALNF;
