@@ -471,3 +471,29 @@ def test_full_grid_n2_tiled_tb(gpu, stencil, oc):
     del x
     torch.cuda.empty_cache()
     assert _relerr(got, ref) <= TOL[dtype], (stencil, oc)
+
+
+@pytest.mark.parametrize("env, name, dims, dtype, oc", [
+    ("STENCIL_NO_M8", "heat3d", (26, 70, 136), "f64", "ST_TB_BM_RT_PR"),
+    ("STENCIL_TILED_FULL", "random2d:2:4", (200, 300), "f64", "TB_BM"),
+    ("STENCIL_TILED_FULL", "random3d:2:5", (24, 40, 72), "f64", "TB_CM"),
+    ("STENCIL_TILED_MVX", "star25", (20, 36, 72), "f32", "TB_BM"),
+])
+def test_round2_paths_bitwise_equal_to_round1(gpu, monkeypatch, env, name, dims, dtype, oc):
+    """Round 2's kernel-path choices (8-row TB-RT setting, full-width and
+    2-column k_tiled intermediate tiles) must not change a single bit of the
+    result: every OC follows the canonical FMA order. Each pair is run with the
+    switch that restores the round-1 path, 10 steps, and checked against the
+    oracle too."""
+    acc, c = si.config_stencil(name)
+    u0 = si.make_field(dims, 13, dtype)
+    ref = oracle.sweep(u0, acc, c, 10, dtype=dtype)
+    outs = []
+    for val in (None, "1" if env == "STENCIL_NO_M8" else ("0" if env == "STENCIL_TILED_FULL" else "1")):
+        if val is None:
+            monkeypatch.delenv(env, raising=False)
+        else:
+            monkeypatch.setenv(env, val)
+        outs.append(_run(sm.Plan(dims, acc, c, dtype, oc), u0, dtype, 10))
+    assert _relerr(outs[0], ref) <= TOL[dtype]
+    assert np.array_equal(outs[0], outs[1])
